@@ -1,0 +1,240 @@
+/*
+ * tq.h -- C ABI of the B200 retry-free / arbitrary-n task queue and the
+ * persistent-thread top-down BFS that drives it.
+ *
+ * Method: Troendle, Ta & Jang, "A Specialized Concurrent Queue for
+ * Scheduling Irregular Workloads on GPUs", ICPP 2019.  Citations are to
+ * /root/reference/PAPER.md lines (P:<line>) with section / listing.
+ *
+ * Conventions for every entry point
+ *   - Plain C types only; no exception or C++ type crosses the ABI.
+ *   - Every function returns a tq_status; TQ_OK (0) on success.  Outputs are
+ *     undefined on any non-OK status.
+ *   - `stream` arguments are cudaStream_t values passed as void* (NULL = the
+ *     legacy default stream).
+ *   - Device pointers are CUDA global-memory pointers on the device the object
+ *     was created on.  Where an entry point says "host or device", the
+ *     library inspects the pointer (cudaPointerGetAttributes) and stages host
+ *     buffers through device memory itself.
+ *   - Ownership: the caller owns every buffer it passes in (CSR arrays, output
+ *     arrays); the library owns the queue storage, the BFS state and scratch,
+ *     and frees them in the matching *_destroy.
+ */
+#ifndef TQ_H_
+#define TQ_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    TQ_OK = 0,
+    TQ_ERR_INVALID = -1,     /* bad argument (null pointer, range, size)      */
+    TQ_ERR_CUDA = -2,        /* a CUDA runtime call failed                    */
+    TQ_ERR_NOMEM = -3,       /* device allocation failed                      */
+    TQ_ERR_QUEUE_FULL = -4,  /* queue-full exception: the kernel aborted, no
+                                retry (P:71 fn2; Listing 3 line 25;
+                                P:281 §4.4 "the user can retry the kernel with
+                                a larger queue")                              */
+    TQ_ERR_TIMEOUT = -5,     /* watchdog expired (protects against hangs)     */
+    TQ_ERR_UNSUPPORTED = -6  /* variant / option not available                */
+} tq_status;
+
+/* Queue variants (§5.3).  RF_AN is the paper's queue; the others
+ * are the comparison designs of the evaluation, built in-repo.              */
+typedef enum {
+    TQ_VARIANT_RF_AN = 0,          /* retry-free + arbitrary-n: proxy lane, one
+                                      64-bit atomicAdd per warp op (P:155,
+                                      P:167-171, Listings 1 and 3)           */
+    TQ_VARIANT_PER_THREAD_AFA = 1, /* retry-free, no proxy: every lane issues
+                                      its own atomicAdd (north-star comparator) */
+    TQ_VARIANT_CAS_RETRY = 2,      /* BASE: traditional lock-free CAS queue,
+                                      one slot per CAS, retries on CAS failure
+                                      and on empty            */
+    TQ_VARIANT_AN = 3,             /* AN: BASE + arbitrary-n (proxy CAS loop
+                                      reserving n slots)             */
+    TQ_VARIANT_ATOMIC_CEILING = 4  /* tq_bench only: proxy atomicAdd on Rear
+                                      with no slot traffic -> R_atom          */
+} tq_variant;
+
+/* ------------------------------------------------------------------------ */
+/* Queue object                                                              */
+/* ------------------------------------------------------------------------ */
+
+/* A bounded circular array of C = 2^k slots (§3.1, Fig 2) with
+ * Front / Rear counters.  Each slot is 8 bytes
+ * {item:32 (high) | seq:32 (low)}; seq replaces the data-not-arrived sentinel
+ * (§4) and the bounds check of Listing 2: for ticket t the slot
+ * is t mod C, seq == (uint32)t means "empty, waiting for ticket t" (dna),
+ * seq == (uint32)(t+1) means "item for ticket t has arrived".  Front, Rear
+ * and Done are monotonic 64-bit tickets.  Requires 2 <= C <= 2^31. */
+typedef struct tq_queue tq_queue;
+
+/* Allocate a queue of at least `capacity` slots (rounded up to a power of
+ * two; capacity < 2 or > 2^31 -> TQ_ERR_INVALID) on CUDA device `device`,
+ * initialised empty.  *out receives the handle. */
+tq_status tq_create(uint64_t capacity, int device, tq_queue **out);
+
+/* Free the queue.  NULL-safe. */
+tq_status tq_destroy(tq_queue *q);
+
+/* Reset to the empty state (every slot dna for lap 0, Front = Rear = Done =
+ * 0, status running) on `stream`; required after a queue-full abort or a
+ * timeout, which can leave slots written but untaken. */
+tq_status tq_reset(tq_queue *q, void *stream);
+
+/* Queue status words (replicated; see tq_device.cuh). */
+enum { TQ_RUNNING = 0, TQ_FINISHED = 1, TQ_ABORTED_FULL = 2, TQ_ABORTED_TIMEOUT = 3 };
+
+/* Raw device view for user kernels that call the device-side operations in
+ * include/tq_device.cuh.  All pointers are device pointers owned by the
+ * queue.  `status` points at TQ_STATUS_COPIES replicas spaced 32 words
+ * apart. */
+typedef struct {
+    unsigned long long *slots;  /* C slots                                  */
+    unsigned long long *front;  /* Front ticket (dequeue reservations)      */
+    unsigned long long *rear;   /* Rear ticket (enqueue reservations)       */
+    unsigned long long *done;   /* completed tasks (termination detection)  */
+    unsigned int *status;       /* TQ_RUNNING / FINISHED / ABORTED_*        */
+    unsigned long long mask;    /* C - 1                                    */
+    unsigned int log2_capacity; /* k                                        */
+    unsigned int reserved_;
+} tq_device_view;
+
+tq_status tq_device_view_get(const tq_queue *q, tq_device_view *out);
+
+/* Host-side copy of the counters (synchronous). */
+typedef struct {
+    uint64_t front, rear, done;
+    uint32_t status;
+} tq_counters;
+tq_status tq_counters_get(const tq_queue *q, tq_counters *out);
+
+/* ------------------------------------------------------------------------ */
+/* Top-down persistent-thread BFS (Algorithm 1; §5.1)        */
+/* ------------------------------------------------------------------------ */
+
+/* Undirected graph as a symmetric CSR with ascending rows, no self loops or
+ * duplicates (the paper's Nodes[]/Edges[], Listing 2).
+ * row_ptr: int64[n_vertices + 1], col: int32[nnz]; 1 <= n_vertices < 2^31.
+ * Pointers are host or device (see the entry point). */
+typedef struct {
+    int64_t n_vertices;
+    int64_t nnz;
+    const int64_t *row_ptr;
+    const int32_t *col;
+} tq_csr;
+
+/* Options; a zero-initialised struct selects every default. */
+typedef struct {
+    uint64_t capacity;  /* queue slots; 0 = 2^ceil(log2(2V)), at least 2^16   */
+    int threads;        /* persistent threads; 0 = SMs x occupancy (P:63,
+                           P:83 "just enough threads to saturate")           */
+    int block;          /* threads per block; 0 = 256                        */
+    int chunk;          /* sub-task size: max edges per task token (P:153
+                           "a fixed number of uniformly complex sub-tasks";
+                           P:159 fn3).  Vertices with more edges are split
+                           into chunk tokens.  0 = 256; power of 2 in
+                           [32, 2^16]                                        */
+    int variant;        /* tq_variant (RF_AN, PER_THREAD_AFA, CAS_RETRY, AN) */
+    void *stream;       /* cudaStream_t                                      */
+    double timeout_s;   /* watchdog; 0 = 60 s                                */
+    int backoff_ns;     /* max idle back-off per empty work cycle; 0 = 256,
+                           < 0 = none                                        */
+    int device;         /* CUDA device for bfs_plan_create / host-pointer runs;
+                           ignored when the CSR is device memory             */
+} bfs_opts;
+
+/* Per-run statistics (device counters, summed over warps). */
+typedef struct {
+    double ms;                  /* device time: init + persistent + unpack     */
+    double ms_kernel;           /* persistent kernel alone                     */
+    uint64_t traversed_edges;   /* undirected edges with a reached endpoint     */
+    uint64_t reached;           /* vertices with level >= 0                    */
+    uint64_t tasks;             /* task tokens processed (vertex + chunk)      */
+    uint64_t chunk_tasks;       /* of which chunk tokens                       */
+    uint64_t edges_scanned;     /* CSR entries examined                        */
+    uint64_t min_atomics;       /* atomicMin issued on W (prefilter passed)    */
+    uint64_t reenqueues;        /* vertices re-enqueued after a level decrease */
+    uint64_t queue_atomics;     /* atomics on Front/Rear/Done (incl. failed CAS) */
+    uint64_t cas_failures;      /* CAS variants only                           */
+    uint64_t empty_polls;       /* work cycles that found no data              */
+    uint64_t tickets;           /* tasks enqueued (Rear advance)               */
+    int32_t max_level;
+    int32_t persistent_threads;
+} bfs_stats;
+
+/* Single-source BFS.  level_out[v] = hop distance from root (-1 unreached);
+ * parent_out[v] = the smallest-id neighbour one level closer to the root
+ * (parent_out[root] = root, -1 unreached).  Either output may be NULL.
+ * Graph and outputs: host or device pointers (device pointers must be on the
+ * current device).  Synchronous.  Returns TQ_ERR_QUEUE_FULL if the queue
+ * overflowed (retry with a larger opts->capacity). */
+tq_status bfs_run(const tq_csr *g, int32_t root, int32_t *level_out, int32_t *parent_out);
+tq_status bfs_run_ex(const tq_csr *g, int32_t root, int32_t *level_out, int32_t *parent_out,
+                     const bfs_opts *opts, bfs_stats *stats);
+
+/* Plans: all application data "must be allocated statically before kernel
+ * launch" (§3.1).  A plan holds a device copy / view of the graph, the
+ * queue, the per-vertex state W and the chunk table, so that repeated runs
+ * (multi-root batches) pay no allocation.  If g's pointers are host memory
+ * the plan copies the graph to the device once; device pointers are used in
+ * place and must outlive the plan. */
+typedef struct bfs_plan bfs_plan;
+tq_status bfs_plan_create(const tq_csr *g, const bfs_opts *opts, bfs_plan **out);
+/* level_out / parent_out: DEVICE pointers (or NULL). Stream-ordered on
+ * opts->stream, but synchronous (it reads the status word back). */
+tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,
+                       bfs_stats *stats);
+tq_status bfs_plan_destroy(bfs_plan *p);
+
+/* ------------------------------------------------------------------------ */
+/* Queue micro-benchmark (BASELINE.json configs[1]; Fig 4 / Fig 5 analogue)  */
+/* ------------------------------------------------------------------------ */
+
+typedef struct {
+    int variant;        /* tq_variant                                         */
+    int warps;          /* persistent warps; 0 = SMs x occupancy              */
+    int batch;          /* items per warp operation b, 1..32                 */
+    uint64_t items;     /* total items N (rounded down to warps*batch*iters)  */
+    uint64_t capacity;  /* queue slots                                        */
+    int work_iters;     /* synthetic ALU work per consumed item               */
+    uint64_t seed;      /* item ids = item_of(seed, g) (inputs/items.py)      */
+    int log_mode;       /* 1: record ticket -> item logs (enq_log/deq_log)    */
+    uint32_t *enq_log;  /* device uint32[items] or NULL                       */
+    uint32_t *deq_log;  /* device uint32[items] or NULL                       */
+    void *stream;
+    double timeout_s;   /* 0 = 60 s                                           */
+    int device;
+} tq_bench_cfg;
+
+typedef struct {
+    double ms;
+    uint64_t items;           /* items actually pushed through                */
+    uint64_t enq, deq;        /* successful enqueues / dequeues               */
+    uint64_t atomics;         /* global atomics on Front/Rear (incl. failed CAS) */
+    uint64_t cas_failures;
+    uint64_t empty_retries;   /* polls / dequeue attempts that found no data  */
+    uint64_t sum_enq, sum_deq, xor_enq, xor_deq; /* fingerprints of splitmix64(item) */
+    int32_t warps;
+    tq_status status;
+} tq_bench_result;
+
+tq_status tq_bench(const tq_bench_cfg *cfg, tq_bench_result *res);
+
+/* ------------------------------------------------------------------------ */
+/* Misc                                                                      */
+/* ------------------------------------------------------------------------ */
+const char *tq_strerror(tq_status s);
+/* Occupancy-derived persistent thread count for the BFS kernel of `variant`
+ * with `block` threads per block on `device`. */
+tq_status tq_persistent_threads(int variant, int block, int device, int *threads_out);
+/* Library version string. */
+const char *tq_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TQ_H_ */

@@ -1,0 +1,11 @@
+"""B200-native retry-free, arbitrary-n task queue and persistent-thread BFS.
+
+Troendle, Ta & Jang, "A Specialized Concurrent Queue for Scheduling Irregular
+Workloads on GPUs", ICPP 2019. The product is `libtq.so` (CUDA for sm_100a
+behind the C ABI in include/tq.h); this package is its thin Python binding.
+"""
+from .api import (BfsPlan, Queue, TQError, VARIANTS, bfs, persistent_threads, queue_bench,
+                  version)
+
+__all__ = ["BfsPlan", "Queue", "TQError", "VARIANTS", "bfs", "persistent_threads", "queue_bench",
+           "version"]

@@ -1,0 +1,54 @@
+"""Build the in-tree shared libraries with nvcc for sm_100a.
+
+libtq.so    <- csrc/*.cu           (the product: kernels + C ABI of include/tq.h)
+
+The .so lands next to this file so it travels with the repo snapshot to the
+GPU box (git-ignored, not gpurun-ignored).
+"""
+from __future__ import annotations
+
+import glob
+import os
+import subprocess
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(HERE)
+LIB = os.path.join(HERE, "libtq.so")
+NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
+         "-shared", "-diag-suppress", "128"]
+
+
+def sources() -> list[str]:
+    return sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu")))
+
+
+def deps() -> list[str]:
+    return (sources() + glob.glob(os.path.join(HERE, "csrc", "*.cuh"))
+            + glob.glob(os.path.join(ROOT, "include", "*")))
+
+
+def up_to_date(lib: str, inputs: list[str]) -> bool:
+    if not os.path.exists(lib):
+        return False
+    t = os.path.getmtime(lib)
+    return all(os.path.getmtime(d) <= t for d in inputs)
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    if not force and up_to_date(LIB, deps()):
+        return LIB
+    tmp = LIB + f".tmp{os.getpid()}"
+    cmd = [NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), "-o", tmp, *sources()]
+    if verbose:
+        cmd.insert(1, "-Xptxas=-v")
+        print(" ".join(cmd))
+    subprocess.check_call(cmd)
+    os.replace(tmp, LIB)
+    return LIB
+
+
+if __name__ == "__main__":
+    import sys
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

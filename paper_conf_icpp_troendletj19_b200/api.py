@@ -1,0 +1,235 @@
+"""Python binding of the tq C ABI (include/tq.h): argument marshalling only.
+
+Every step of the hot path runs in libtq.so's CUDA kernels; this module only
+turns torch tensors / numpy arrays into pointers and status codes into
+exceptions. PyTorch is used for device memory and streams.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Optional
+
+import numpy as np
+
+from . import _lib
+from ._lib import TQError, VARIANTS, check, lib
+
+__all__ = ["bfs", "BfsPlan", "Queue", "queue_bench", "persistent_threads", "TQError", "VARIANTS",
+           "version"]
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _is_tensor(x) -> bool:
+    try:
+        import torch
+        return isinstance(x, torch.Tensor)
+    except ImportError:  # pragma: no cover
+        return False
+
+
+def _ptr(x) -> Optional[int]:
+    if x is None:
+        return None
+    if _is_tensor(x):
+        if not x.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        return x.data_ptr()
+    if isinstance(x, np.ndarray):
+        if not x.flags.c_contiguous:
+            raise ValueError("array must be C-contiguous")
+        return x.ctypes.data
+    raise TypeError(f"expected a torch.Tensor or numpy.ndarray, got {type(x)}")
+
+
+def _variant(v) -> int:
+    if isinstance(v, str):
+        return VARIANTS[v]
+    return int(v)
+
+
+def _stream_ptr(stream, like=None) -> Optional[int]:
+    if stream is not None:
+        return stream if isinstance(stream, int) else stream.cuda_stream
+    if like is not None and _is_tensor(like) and like.is_cuda:
+        torch = _torch()
+        return torch.cuda.current_stream(like.device).cuda_stream
+    return None
+
+
+def _csr(row_ptr, col) -> _lib.tq_csr:
+    n = int(row_ptr.shape[0]) - 1
+    nnz = int(col.shape[0])
+    if _is_tensor(row_ptr):
+        torch = _torch()
+        if row_ptr.dtype != torch.int64 or col.dtype != torch.int32:
+            raise TypeError("row_ptr must be int64 and col int32")
+    else:
+        if row_ptr.dtype != np.int64 or col.dtype != np.int32:
+            raise TypeError("row_ptr must be int64 and col int32")
+    return _lib.tq_csr(n, nnz, _ptr(row_ptr), _ptr(col))
+
+
+def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None, timeout_s=0.0,
+          backoff_ns=0, device=0) -> _lib.bfs_opts:
+    return _lib.bfs_opts(int(capacity), int(threads), int(block), int(chunk), _variant(variant),
+                         stream, float(timeout_s), int(backoff_ns), int(device))
+
+
+def _stats_dict(st: _lib.bfs_stats) -> dict:
+    return {f: getattr(st, f) for f, _ in st._fields_}
+
+
+def _empty_like_graph(row_ptr, n):
+    if _is_tensor(row_ptr):
+        torch = _torch()
+        return torch.empty(n, dtype=torch.int32, device=row_ptr.device)
+    return np.empty(n, dtype=np.int32)
+
+
+def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool = True,
+        variant="rf_an", capacity: int = 0, threads: int = 0, chunk: int = 0, stream=None,
+        timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0):
+    """One-shot `bfs_run_ex`: returns (level, parent, stats).
+
+    Graph arrays may be CUDA tensors (used in place) or host numpy arrays
+    (staged to the device by the library). Outputs default to the graph's
+    kind of memory.
+    """
+    g = _csr(row_ptr, col)
+    n = g.n_vertices
+    if level is None:
+        level = _empty_like_graph(row_ptr, n)
+    if parent is None and want_parent:
+        parent = _empty_like_graph(row_ptr, n)
+    o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
+              backoff_ns, row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device)
+    st = _lib.bfs_stats()
+    check(lib().bfs_run_ex(ctypes.byref(g), int(root), _ptr(level), _ptr(parent), ctypes.byref(o),
+                           ctypes.byref(st)), "bfs_run_ex")
+    return level, parent, _stats_dict(st)
+
+
+class BfsPlan:
+    """`bfs_plan_create` / `bfs_plan_run` / `bfs_plan_destroy`.
+
+    Static allocation before launch: graph view, queue, W and the
+    chunk table live for the plan's lifetime; `run` only launches.
+    """
+
+    def __init__(self, row_ptr, col, *, variant="rf_an", capacity: int = 0, threads: int = 0,
+                 chunk: int = 0, stream=None, timeout_s: float = 0.0, backoff_ns: int = 0,
+                 device: int = 0):
+        self._keep = (row_ptr, col)  # device arrays must outlive the plan
+        self._g = _csr(row_ptr, col)
+        self.n_vertices = self._g.n_vertices
+        self.nnz = self._g.nnz
+        self.device = row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device
+        o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
+                  backoff_ns, self.device)
+        h = ctypes.c_void_p()
+        check(lib().bfs_plan_create(ctypes.byref(self._g), ctypes.byref(o), ctypes.byref(h)),
+              "bfs_plan_create")
+        self._h = h
+
+    def run(self, root: int, level=None, parent=None) -> dict:
+        st = _lib.bfs_stats()
+        check(lib().bfs_plan_run(self._h, int(root), _ptr(level), _ptr(parent), ctypes.byref(st)),
+              "bfs_plan_run")
+        return _stats_dict(st)
+
+    def close(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            lib().bfs_plan_destroy(h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+class Queue:
+    """A device queue object (`tq_create` ... `tq_destroy`)."""
+
+    def __init__(self, capacity: int, device: int = 0):
+        h = ctypes.c_void_p()
+        check(lib().tq_create(int(capacity), int(device), ctypes.byref(h)), "tq_create")
+        self._h = h
+
+    def reset(self, stream=None):
+        check(lib().tq_reset(self._h, stream), "tq_reset")
+
+    def view(self) -> _lib.tq_device_view:
+        v = _lib.tq_device_view()
+        check(lib().tq_device_view_get(self._h, ctypes.byref(v)), "tq_device_view_get")
+        return v
+
+    def counters(self) -> dict:
+        c = _lib.tq_counters()
+        check(lib().tq_counters_get(self._h, ctypes.byref(c)), "tq_counters_get")
+        return {"front": c.front, "rear": c.rear, "done": c.done, "status": c.status}
+
+    @property
+    def capacity(self) -> int:
+        return int(self.view().mask) + 1
+
+    def close(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            lib().tq_destroy(h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def queue_bench(variant="rf_an", *, warps: int = 0, batch: int = 32, items: int = 1 << 24,
+                capacity: int = 1 << 20, work_iters: int = 0, seed: int = 3, log: bool = False,
+                stream=None, timeout_s: float = 0.0, device: int = 0) -> dict:
+    """`tq_bench`: enqueue/dequeue throughput of one queue variant.
+
+    With log=True returns 'enq_log' / 'deq_log' (ticket -> item, CUDA tensors).
+    """
+    enq_log = deq_log = None
+    if log:
+        torch = _torch()
+        enq_log = torch.zeros(items, dtype=torch.int32, device=f"cuda:{device}")
+        deq_log = torch.zeros(items, dtype=torch.int32, device=f"cuda:{device}")
+    cfg = _lib.tq_bench_cfg(_variant(variant), int(warps), int(batch), int(items), int(capacity),
+                            int(work_iters), int(seed), int(log), _ptr(enq_log), _ptr(deq_log),
+                            _stream_ptr(stream), float(timeout_s), int(device))
+    res = _lib.tq_bench_result()
+    status = lib().tq_bench(ctypes.byref(cfg), ctypes.byref(res))
+    out = {f: getattr(res, f) for f, _ in res._fields_}
+    out["status"] = status
+    if log:
+        out["enq_log"], out["deq_log"] = enq_log, deq_log
+    if status not in (_lib.TQ_OK,):
+        raise TQError(status, "tq_bench")
+    return out
+
+
+def persistent_threads(variant="rf_an", device: int = 0) -> int:
+    t = ctypes.c_int()
+    check(lib().tq_persistent_threads(_variant(variant), 256, int(device), ctypes.byref(t)),
+          "tq_persistent_threads")
+    return t.value
+
+
+def version() -> str:
+    return lib().tq_version().decode()

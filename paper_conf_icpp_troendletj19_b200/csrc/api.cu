@@ -1,0 +1,553 @@
+// api.cu -- implementation of the C ABI declared in include/tq.h.
+//
+// Host-side runtime around the kernels: queue objects (static allocation
+// before launch, §3.1), BFS plans, pointer staging for host buffers,
+// persistent-grid sizing from the occupancy API, event timing,
+// status read-back (queue-full abort -> TQ_ERR_QUEUE_FULL) and the
+// queue micro-benchmark driver.
+#include <math.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <new>
+
+#include "internal.cuh"
+
+using namespace tqk;
+
+#define TQ_VERSION_STRING "tq-b200 0.1 (sm_100a)"
+
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = true;
+    explicit DeviceGuard(int dev)
+    {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (dev >= 0 && dev != prev) ok = cudaSetDevice(dev) == cudaSuccess;
+    }
+    ~DeviceGuard()
+    {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+tq_status from_cuda(cudaError_t e)
+{
+    if (e == cudaSuccess) return TQ_OK;
+    cudaGetLastError();  // clear sticky-free errors
+    if (e == cudaErrorMemoryAllocation) return TQ_ERR_NOMEM;
+    return TQ_ERR_CUDA;
+}
+
+#define CK(call)                                        \
+    do {                                                \
+        cudaError_t e_ = (call);                        \
+        if (e_ != cudaSuccess) return from_cuda(e_);    \
+    } while (0)
+
+// Returns 1 for device (or managed) memory, 0 for host memory, -1 on error.
+int is_device_ptr(const void *p, int *device)
+{
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+        if (device) *device = a.device;
+        return 1;
+    }
+    return 0;
+}
+
+uint64_t next_pow2(uint64_t x)
+{
+    uint64_t c = 1;
+    while (c < x) c <<= 1;
+    return c;
+}
+
+int sm_count(int dev)
+{
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return sms > 0 ? sms : 1;
+}
+
+// counter block layout (bytes): Front, Rear, Done 4 KiB apart (separate L2
+// lines and slices); status replicas 128 B apart after them.
+constexpr size_t kOffFront = 0, kOffRear = 4096, kOffDone = 8192, kOffStatus = 12288;
+constexpr size_t kCtrBytes = kOffStatus + TQ_STATUS_COPIES * TQ_STATUS_STRIDE * sizeof(unsigned);
+
+}  // namespace
+
+struct tq_queue {
+    int device = 0;
+    uint64_t cap = 0;
+    unsigned log2cap = 0;
+    unsigned long long *slots = nullptr;
+    char *ctr = nullptr;
+    tq_device_view view{};
+};
+
+struct bfs_plan {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    int variant = 0, block = 256, blocks = 0, chunk = 256, backoff_ns = 256;
+    double timeout_s = 60.0;
+    int64_t n = 0, nnz = 0;
+    int64_t *row_ptr = nullptr;
+    int32_t *col = nullptr;
+    bool owns_graph = false;
+    unsigned long long *W = nullptr;
+    int32_t *hub_base = nullptr;
+    int2 *chunk_tab = nullptr;
+    int64_t n_chunks = 0;
+    tq_queue *q = nullptr;
+    unsigned long long *stats = nullptr;      // device, kStatCount
+    unsigned long long *stats_h = nullptr;    // pinned
+    unsigned long long next_ticket = 0;
+    bool dirty = false;
+    int32_t *out_scratch = nullptr;           // for host outputs
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+};
+
+extern "C" {
+
+const char *tq_version(void) { return TQ_VERSION_STRING; }
+
+const char *tq_strerror(tq_status s)
+{
+    switch (s) {
+    case TQ_OK: return "ok";
+    case TQ_ERR_INVALID: return "invalid argument";
+    case TQ_ERR_CUDA: return "CUDA error";
+    case TQ_ERR_NOMEM: return "out of device memory";
+    case TQ_ERR_QUEUE_FULL: return "queue full: kernel aborted (retry with a larger queue)";
+    case TQ_ERR_TIMEOUT: return "watchdog timeout";
+    case TQ_ERR_UNSUPPORTED: return "unsupported";
+    default: return "unknown status";
+    }
+}
+
+// ------------------------------------------------------------------------
+// queue objects
+// ------------------------------------------------------------------------
+tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
+{
+    if (!out) return TQ_ERR_INVALID;
+    *out = nullptr;
+    if (capacity < 2 || capacity > (1ull << 31)) return TQ_ERR_INVALID;
+    DeviceGuard g(device);
+    if (!g.ok) return TQ_ERR_INVALID;
+    tq_queue *q = new (std::nothrow) tq_queue;
+    if (!q) return TQ_ERR_NOMEM;
+    q->device = device;
+    q->cap = next_pow2(capacity);
+    while ((1ull << q->log2cap) < q->cap) ++q->log2cap;
+    cudaError_t e = cudaMalloc(&q->slots, q->cap * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc(&q->ctr, kCtrBytes);
+    if (e != cudaSuccess) {
+        cudaFree(q->slots);
+        delete q;
+        return from_cuda(e);
+    }
+    q->view.slots = q->slots;
+    q->view.front = (unsigned long long *)(q->ctr + kOffFront);
+    q->view.rear = (unsigned long long *)(q->ctr + kOffRear);
+    q->view.done = (unsigned long long *)(q->ctr + kOffDone);
+    q->view.status = (unsigned *)(q->ctr + kOffStatus);
+    q->view.mask = q->cap - 1;
+    q->view.log2_capacity = q->log2cap;
+    tq_status st = tq_reset(q, nullptr);
+    if (st == TQ_OK) st = from_cuda(cudaDeviceSynchronize());
+    if (st != TQ_OK) {
+        tq_destroy(q);
+        return st;
+    }
+    *out = q;
+    return TQ_OK;
+}
+
+tq_status tq_destroy(tq_queue *q)
+{
+    if (!q) return TQ_OK;
+    DeviceGuard g(q->device);
+    cudaFree(q->slots);
+    cudaFree(q->ctr);
+    delete q;
+    return TQ_OK;
+}
+
+tq_status tq_reset(tq_queue *q, void *stream)
+{
+    if (!q) return TQ_ERR_INVALID;
+    DeviceGuard g(q->device);
+    CK(cudaMemsetAsync(q->ctr, 0, kCtrBytes, (cudaStream_t)stream));
+    CK(launch_queue_reset(q->view, (cudaStream_t)stream));
+    return TQ_OK;
+}
+
+tq_status tq_device_view_get(const tq_queue *q, tq_device_view *out)
+{
+    if (!q || !out) return TQ_ERR_INVALID;
+    *out = q->view;
+    return TQ_OK;
+}
+
+tq_status tq_counters_get(const tq_queue *q, tq_counters *out)
+{
+    if (!q || !out) return TQ_ERR_INVALID;
+    DeviceGuard g(q->device);
+    unsigned long long f = 0, r = 0, d = 0;
+    unsigned s = 0;
+    CK(cudaMemcpy(&f, q->view.front, 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&r, q->view.rear, 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&d, q->view.done, 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&s, q->view.status, 4, cudaMemcpyDeviceToHost));
+    out->front = f;
+    out->rear = r;
+    out->done = d;
+    out->status = s;
+    return TQ_OK;
+}
+
+tq_status tq_persistent_threads(int variant, int block, int device, int *threads_out)
+{
+    if (!threads_out) return TQ_ERR_INVALID;
+    if (block == 0) block = 256;
+    DeviceGuard g(device);
+    int per_sm = 0;
+    if (bfs_occupancy(variant, block, &per_sm) != cudaSuccess) {
+        cudaGetLastError();
+        return TQ_ERR_INVALID;
+    }
+    *threads_out = per_sm * sm_count(device) * block;
+    return TQ_OK;
+}
+
+// ------------------------------------------------------------------------
+// BFS plans
+// ------------------------------------------------------------------------
+tq_status bfs_plan_destroy(bfs_plan *p)
+{
+    if (!p) return TQ_OK;
+    DeviceGuard g(p->device);
+    if (p->stream) cudaStreamSynchronize(p->stream);
+    for (auto &e : p->ev)
+        if (e) cudaEventDestroy(e);
+    if (p->owns_graph) {
+        cudaFree(p->row_ptr);
+        cudaFree(p->col);
+    }
+    cudaFree(p->W);
+    cudaFree(p->hub_base);
+    cudaFree(p->chunk_tab);
+    cudaFree(p->stats);
+    cudaFree(p->out_scratch);
+    if (p->stats_h) cudaFreeHost(p->stats_h);
+    tq_destroy(p->q);
+    delete p;
+    return TQ_OK;
+}
+
+tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **out)
+{
+    if (!gph || !out) return TQ_ERR_INVALID;
+    *out = nullptr;
+    bfs_opts o;
+    memset(&o, 0, sizeof(o));
+    if (opts) o = *opts;
+    const int64_t n = gph->n_vertices, nnz = gph->nnz;
+    if (n < 1 || n >= (1ll << 31) || nnz < 0 || !gph->row_ptr || (nnz > 0 && !gph->col))
+        return TQ_ERR_INVALID;
+    if (o.variant < TQ_VARIANT_RF_AN || o.variant > TQ_VARIANT_AN) return TQ_ERR_UNSUPPORTED;
+    int chunk = o.chunk ? o.chunk : 256;
+    if (chunk < 32 || chunk > 65536 || (chunk & (chunk - 1))) return TQ_ERR_INVALID;
+    const int block = o.block ? o.block : 256;
+    if (block != 256) return TQ_ERR_UNSUPPORTED;
+
+    int gdev = o.device;
+    const int dev_graph = is_device_ptr(gph->row_ptr, &gdev);
+    if (dev_graph && nnz > 0 && !is_device_ptr(gph->col, nullptr)) return TQ_ERR_INVALID;
+    DeviceGuard g(gdev);
+    if (!g.ok) return TQ_ERR_INVALID;
+
+    bfs_plan *p = new (std::nothrow) bfs_plan;
+    if (!p) return TQ_ERR_NOMEM;
+    p->device = gdev;
+    p->stream = (cudaStream_t)o.stream;
+    p->variant = o.variant;
+    p->block = block;
+    p->chunk = chunk;
+    p->backoff_ns = o.backoff_ns == 0 ? 256 : (o.backoff_ns < 0 ? 0 : o.backoff_ns);
+    p->timeout_s = o.timeout_s > 0 ? o.timeout_s : 60.0;
+    p->n = n;
+    p->nnz = nnz;
+
+    auto fail = [&](tq_status s) {
+        bfs_plan_destroy(p);
+        return s;
+    };
+    cudaError_t e;
+    if (dev_graph) {
+        p->row_ptr = const_cast<int64_t *>(gph->row_ptr);
+        p->col = const_cast<int32_t *>(gph->col);
+    } else {
+        p->owns_graph = true;
+        e = cudaMalloc(&p->row_ptr, (size_t)(n + 1) * sizeof(int64_t));
+        if (e == cudaSuccess) e = cudaMalloc(&p->col, (size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t));
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(p->row_ptr, gph->row_ptr, (size_t)(n + 1) * sizeof(int64_t),
+                                cudaMemcpyHostToDevice, p->stream);
+        if (e == cudaSuccess && nnz > 0)
+            e = cudaMemcpyAsync(p->col, gph->col, (size_t)nnz * sizeof(int32_t),
+                                cudaMemcpyHostToDevice, p->stream);
+        if (e != cudaSuccess) return fail(from_cuda(e));
+    }
+    e = cudaMalloc(&p->W, (size_t)n * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc(&p->hub_base, (size_t)n * sizeof(int32_t));
+    if (e == cudaSuccess) e = cudaMalloc(&p->stats, kStatCount * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
+    for (auto &ev : p->ev)
+        if (e == cudaSuccess) e = cudaEventCreate(&ev);
+    if (e != cudaSuccess) return fail(from_cuda(e));
+    e = build_chunk_table(p->row_ptr, n, chunk, p->hub_base, &p->chunk_tab, &p->n_chunks, p->stream);
+    if (e != cudaSuccess) return fail(from_cuda(e));
+    if (n + p->n_chunks >= (1ll << 31)) return fail(TQ_ERR_UNSUPPORTED);
+
+    uint64_t cap = o.capacity ? o.capacity : next_pow2((uint64_t)(2 * n));
+    if (!o.capacity && cap < (1ull << 16)) cap = 1ull << 16;
+    tq_status st = tq_create(cap, gdev, &p->q);
+    if (st != TQ_OK) return fail(st);
+
+    int per_sm = 0;
+    e = bfs_occupancy(p->variant, block, &per_sm);
+    if (e != cudaSuccess) return fail(from_cuda(e));
+    const int full = per_sm * sm_count(gdev);
+    if (o.threads > 0) {
+        p->blocks = (o.threads + block - 1) / block;
+    } else {
+        p->blocks = full;
+    }
+    if (p->blocks < 1) p->blocks = 1;
+    e = cudaStreamSynchronize(p->stream);
+    if (e != cudaSuccess) return fail(from_cuda(e));
+    *out = p;
+    return TQ_OK;
+}
+
+static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int32_t *parent,
+                                 bfs_stats *stats)
+{
+    cudaStream_t s = p->stream;
+    if (p->dirty) {
+        tq_status st = tq_reset(p->q, s);
+        if (st != TQ_OK) return st;
+        p->next_ticket = 0;
+        p->dirty = false;
+    }
+    BfsParams bp{};
+    bp.q = p->q->view;
+    bp.row_ptr = p->row_ptr;
+    bp.col = p->col;
+    bp.W = p->W;
+    bp.chunk_tab = p->chunk_tab;
+    bp.hub_base = p->hub_base;
+    bp.stats = p->stats;
+    bp.n_vertices = p->n;
+    bp.chunk = p->chunk;
+    bp.backoff_ns = p->backoff_ns;
+    bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
+
+    CK(cudaEventRecord(p->ev[0], s));
+    CK(launch_bfs_init(bp, root, p->next_ticket, s));
+    CK(cudaEventRecord(p->ev[1], s));
+    CK(launch_bfs_persistent(p->variant, bp, p->blocks, p->block, s));
+    CK(cudaEventRecord(p->ev[2], s));
+    CK(launch_bfs_unpack(bp, level, parent, s));
+    CK(cudaEventRecord(p->ev[3], s));
+    CK(cudaMemcpyAsync(p->stats_h, p->stats, kStatCount * sizeof(unsigned long long),
+                       cudaMemcpyDeviceToHost, s));
+    unsigned long long ctr[3] = {0, 0, 0};
+    unsigned status = 0;
+    CK(cudaMemcpyAsync(&ctr[0], p->q->view.front, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&ctr[1], p->q->view.rear, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&ctr[2], p->q->view.done, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&status, p->q->view.status, 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+
+    const unsigned long long t0 = p->next_ticket;
+    if (status == TQ_FINISHED) {
+        // every reserved ticket below Rear was taken; slots of tickets
+        // [Rear, Rear + C) all hold "empty for t", so the next run can start
+        // at Rear without an O(C) reset
+        p->next_ticket = ctr[1];
+    } else {
+        p->dirty = true;
+    }
+    if (stats) {
+        memset(stats, 0, sizeof(*stats));
+        float a = 0, b = 0;
+        cudaEventElapsedTime(&a, p->ev[0], p->ev[3]);
+        cudaEventElapsedTime(&b, p->ev[1], p->ev[2]);
+        stats->ms = a;
+        stats->ms_kernel = b;
+        const unsigned long long *h = p->stats_h;
+        stats->tasks = h[ST_TASKS];
+        stats->chunk_tasks = h[ST_CHUNK_TASKS];
+        stats->edges_scanned = h[ST_EDGES];
+        stats->min_atomics = h[ST_MIN_ATOMICS];
+        stats->reenqueues = h[ST_REENQUEUES];
+        stats->queue_atomics = h[ST_QUEUE_ATOMICS];
+        stats->cas_failures = h[ST_CAS_FAILURES];
+        stats->empty_polls = h[ST_EMPTY_POLLS];
+        stats->reached = h[ST_REACHED];
+        stats->traversed_edges = h[ST_DEG_SUM] / 2;
+        stats->max_level = (int32_t)h[ST_MAX_LEVEL];
+        stats->tickets = ctr[1] - t0;
+        stats->persistent_threads = p->blocks * p->block;
+    }
+    if (status == TQ_FINISHED) return TQ_OK;
+    if (status == TQ_ABORTED_FULL) return TQ_ERR_QUEUE_FULL;
+    if (status == TQ_ABORTED_TIMEOUT) return TQ_ERR_TIMEOUT;
+    return TQ_ERR_CUDA;
+}
+
+tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,
+                       bfs_stats *stats)
+{
+    if (!p || root < 0 || root >= p->n) return TQ_ERR_INVALID;
+    DeviceGuard g(p->device);
+    const bool host_l = level_out && !is_device_ptr(level_out, nullptr);
+    const bool host_p = parent_out && !is_device_ptr(parent_out, nullptr);
+    if (!host_l && !host_p) return plan_run_device(p, root, level_out, parent_out, stats);
+    if (!p->out_scratch) CK(cudaMalloc(&p->out_scratch, (size_t)p->n * 2 * sizeof(int32_t)));
+    int32_t *dl = level_out ? (host_l ? p->out_scratch : level_out) : nullptr;
+    int32_t *dp = parent_out ? (host_p ? p->out_scratch + p->n : parent_out) : nullptr;
+    tq_status st = plan_run_device(p, root, dl, dp, stats);
+    if (st != TQ_OK) return st;
+    if (host_l)
+        CK(cudaMemcpyAsync(level_out, dl, (size_t)p->n * sizeof(int32_t), cudaMemcpyDeviceToHost, p->stream));
+    if (host_p)
+        CK(cudaMemcpyAsync(parent_out, dp, (size_t)p->n * sizeof(int32_t), cudaMemcpyDeviceToHost, p->stream));
+    CK(cudaStreamSynchronize(p->stream));
+    return TQ_OK;
+}
+
+tq_status bfs_run_ex(const tq_csr *g, int32_t root, int32_t *level_out, int32_t *parent_out,
+                     const bfs_opts *opts, bfs_stats *stats)
+{
+    if (!g || root < 0 || root >= g->n_vertices) return TQ_ERR_INVALID;
+    bfs_plan *p = nullptr;
+    tq_status st = bfs_plan_create(g, opts, &p);
+    if (st != TQ_OK) return st;
+    st = bfs_plan_run(p, root, level_out, parent_out, stats);
+    bfs_plan_destroy(p);
+    return st;
+}
+
+tq_status bfs_run(const tq_csr *g, int32_t root, int32_t *level_out, int32_t *parent_out)
+{
+    return bfs_run_ex(g, root, level_out, parent_out, nullptr, nullptr);
+}
+
+// ------------------------------------------------------------------------
+// queue micro-benchmark
+// ------------------------------------------------------------------------
+tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
+{
+    if (!c || !r) return TQ_ERR_INVALID;
+    memset(r, 0, sizeof(*r));
+    if (c->variant < TQ_VARIANT_RF_AN || c->variant > TQ_VARIANT_ATOMIC_CEILING) return TQ_ERR_UNSUPPORTED;
+    if (c->batch < 1 || c->batch > 32 || c->items == 0 || c->warps < 0) return TQ_ERR_INVALID;
+    DeviceGuard g(c->device);
+    if (!g.ok) return TQ_ERR_INVALID;
+    int warps = c->warps;
+    if (warps == 0) {
+        int per_sm = 0;
+        CK(bench_occupancy(c->variant, 256, &per_sm));
+        warps = per_sm * sm_count(c->device) * 8;
+    }
+    int wpb = 8;
+    while (warps % wpb) wpb >>= 1;
+    const int block = 32 * wpb, blocks = warps / wpb;
+    const uint64_t iters = c->items / ((uint64_t)warps * c->batch);
+    if (iters == 0 || iters > (1ull << 30)) return TQ_ERR_INVALID;
+    const uint64_t items = iters * warps * c->batch;
+    if (c->log_mode && (!c->enq_log || !c->deq_log)) return TQ_ERR_INVALID;
+    uint64_t cap = c->capacity ? c->capacity : (1ull << 20);
+    if ((uint64_t)warps * c->batch > next_pow2(cap)) return TQ_ERR_INVALID;  // cannot hold in-flight items
+
+    tq_queue *q = nullptr;
+    tq_status st = tq_create(cap, c->device, &q);
+    if (st != TQ_OK) return st;
+    cudaStream_t s = (cudaStream_t)c->stream;
+    unsigned long long *out = nullptr, out_h[16];
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    cudaError_t e = cudaMalloc(&out, sizeof(out_h));
+    if (e == cudaSuccess) e = cudaMemsetAsync(out, 0, sizeof(out_h), s);
+    if (e == cudaSuccess) e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    BenchParams bp{};
+    bp.q = q->view;
+    bp.batch = c->batch;
+    bp.iters = (int)iters;
+    bp.work_iters = c->work_iters;
+    {
+        // seed32 = low 32 bits of splitmix64(seed) (inputs/items.py:seed32)
+        unsigned long long x = c->seed;
+        x ^= x >> 30; x *= 0xBF58476D1CE4E5B9ull;
+        x ^= x >> 27; x *= 0x94D049BB133111EBull;
+        x ^= x >> 31;
+        bp.seed32 = (uint32_t)x;
+    }
+    bp.enq_log = c->log_mode ? c->enq_log : nullptr;
+    bp.deq_log = c->log_mode ? c->deq_log : nullptr;
+    bp.out = out;
+    bp.timeout_ns = (unsigned long long)((c->timeout_s > 0 ? c->timeout_s : 60.0) * 1e9);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess) e = cudaEventRecord(e0, s);
+    if (e == cudaSuccess) e = launch_bench(c->variant, bp, blocks, block, s);
+    if (e == cudaSuccess) e = cudaEventRecord(e1, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(out_h, out, sizeof(out_h), cudaMemcpyDeviceToHost, s);
+    unsigned status = 0;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&status, q->view.status, 4, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess) {
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        r->ms = ms;
+        r->items = items;
+        r->enq = out_h[0];
+        r->deq = out_h[1];
+        r->atomics = out_h[2];
+        r->cas_failures = out_h[3];
+        r->empty_retries = out_h[4];
+        r->sum_enq = out_h[5];
+        r->sum_deq = out_h[6];
+        r->xor_enq = out_h[7];
+        r->xor_deq = out_h[8];
+        r->warps = warps;
+        if (status == TQ_ABORTED_FULL)
+            st = TQ_ERR_QUEUE_FULL;
+        else if (status == TQ_ABORTED_TIMEOUT)
+            st = TQ_ERR_TIMEOUT;
+        else if (c->variant != TQ_VARIANT_ATOMIC_CEILING && (r->deq != items || r->enq != items))
+            st = TQ_ERR_TIMEOUT;
+    } else {
+        st = from_cuda(e);
+    }
+    r->status = st;
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+    cudaFree(out);
+    tq_destroy(q);
+    return st;
+}
+
+}  // extern "C"

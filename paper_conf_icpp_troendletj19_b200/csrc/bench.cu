@@ -1,0 +1,336 @@
+// bench.cu -- queue micro-benchmark (BASELINE.json configs[1]):
+// every warp repeatedly enqueues `batch` unique items, reserves `batch`
+// dequeue tickets, waits for its items to arrive and consumes them, for the
+// RF/AN queue (Listings 1-3) and the comparison queues
+// (per-thread AFA, CAS-retry BASE, AN).  The retry ratio of
+// Fig 5 is atomics_issued / items.
+#include "internal.cuh"
+
+namespace tqk {
+
+enum BenchOut {
+    BO_ENQ = 0, BO_DEQ, BO_ATOM, BO_FAIL, BO_EMPTY, BO_SUM_ENQ, BO_SUM_DEQ, BO_XOR_ENQ, BO_XOR_DEQ,
+    BO_SINK, BO_COUNT_
+};
+
+// Twin of inputs/items.py:item_of (a bijection on 32-bit integers).
+__device__ __forceinline__ uint32_t item_of(uint32_t seed32, unsigned long long g)
+{
+    uint32_t x = (uint32_t)g ^ seed32;
+    x *= 0x9E3779B1u;
+    x ^= x >> 16;
+    x *= 0x85EBCA6Bu;
+    x ^= x >> 13;
+    return x;
+}
+
+// Twin of inputs/graphs.py:_mix64 (splitmix64 finaliser), item fingerprints.
+__device__ __forceinline__ unsigned long long mix64(unsigned long long x)
+{
+    x ^= x >> 30;
+    x *= 0xBF58476D1CE4E5B9ull;
+    x ^= x >> 27;
+    x *= 0x94D049BB133111EBull;
+    x ^= x >> 31;
+    return x;
+}
+
+__device__ __forceinline__ bool bench_publish(const tq_device_view &q, unsigned long long t, uint32_t item)
+{
+    return tq_publish(q, t, item);
+}
+
+// BASE enqueue / dequeue with the ticket returned (for the logs)
+__device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t item,
+                                              unsigned long long *t_out, unsigned *atom, unsigned *fail)
+{
+    for (;;) {
+        const unsigned long long pos = tq_ld_relaxed(q.rear);
+        unsigned long long *s = q.slots + (pos & q.mask);
+        const unsigned long long v = tq_ld_relaxed(s);
+        const int dif = (int)((unsigned)v - (unsigned)pos);
+        if (dif == 0) {
+            ++*atom;
+            if (tq_atom_cas(q.rear, pos, pos + 1) == pos) {
+                tq_st_relaxed(s, ((unsigned long long)item << 32) | (unsigned)(pos + 1));
+                *t_out = pos;
+                return true;
+            }
+            ++*fail;
+        } else if (dif < 0) {
+            tq_status_set_thread(q, TQ_ABORTED_FULL);
+            return false;
+        }
+    }
+}
+
+__device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *item,
+                                             unsigned long long *t_out, unsigned *atom, unsigned *fail)
+{
+    for (;;) {
+        const unsigned long long pos = tq_ld_relaxed(q.front);
+        unsigned long long *s = q.slots + (pos & q.mask);
+        const unsigned long long v = tq_ld_relaxed(s);
+        const int dif = (int)((unsigned)v - (unsigned)(pos + 1));
+        if (dif == 0) {
+            ++*atom;
+            if (tq_atom_cas(q.front, pos, pos + 1) == pos) {
+                *item = (uint32_t)(v >> 32);
+                tq_st_relaxed(s, (unsigned long long)(unsigned)(pos + q.mask + 1));
+                *t_out = pos;
+                return 1;
+            }
+            ++*fail;
+        } else if (dif < 0) {
+            return 0;
+        }
+    }
+}
+
+// polled every 1024 empty spins: watchdog + abort propagation
+__device__ __noinline__ bool should_stop(const tq_device_view &q, unsigned warp, unsigned long long deadline)
+{
+    if (tq_globaltimer() > deadline) tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
+    return tq_status_read(q, warp) != TQ_RUNNING;
+}
+
+template <int VARIANT>
+__global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
+{
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long warp_gid = ((unsigned long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const tq_device_view q = p.q;
+    const unsigned long long cap = q.mask + 1;
+    const bool active = (int)lane < p.batch;
+    unsigned n_enq = 0, n_deq = 0, atom = 0, fail = 0, empty = 0;
+    unsigned long long s_enq = 0, s_deq = 0, x_enq = 0, x_deq = 0, sink = 0;
+    const unsigned long long deadline = tq_globaltimer() + p.timeout_ns;
+    bool stop = false;
+
+    for (int it = 0; it < p.iters && !stop; ++it) {
+        const unsigned long long g = (warp_gid * (unsigned long long)p.iters + it) * p.batch + lane;
+        const uint32_t item = item_of(p.seed32, g);
+
+        if constexpr (VARIANT == TQ_VARIANT_ATOMIC_CEILING) {
+            if (lane == 0) {
+                sink += tq_atom_add(q.rear, (unsigned long long)p.batch);
+                ++atom;
+            }
+            if (active) {
+                ++n_enq;
+                ++n_deq;
+            }
+            continue;
+        } else {
+            // ------------------------------ enqueue ------------------------------
+            unsigned long long et = 0;
+            bool eok = true;
+            if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
+                const unsigned long long base = tq_warp_reserve_rear(q, (unsigned)p.batch, &atom);
+                et = base + lane;
+                if (active) eok = bench_publish(q, et, item);
+            } else if constexpr (VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
+                if (active) {
+                    et = tq_atom_add(q.rear, 1ull);
+                    ++atom;
+                    eok = bench_publish(q, et, item);
+                }
+            } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
+                if (active) eok = b_cas_enqueue(q, item, &et, &atom, &fail);
+            } else {  // AN: proxy CAS loop reserving `batch` slots
+                unsigned long long base = 0;
+                // reuse the BFS AN reservation logic inline
+                for (;;) {
+                    unsigned long long pos = 0;
+                    if (lane == 0) pos = tq_ld_relaxed(q.rear);
+                    pos = tq_shfl64(pos, 0);
+                    int dif = 0;
+                    if (active) dif = (int)((unsigned)tq_ld_relaxed(q.slots + ((pos + lane) & q.mask)) -
+                                            (unsigned)(pos + lane));
+                    if (__any_sync(TQ_FULL_MASK, dif > 0)) continue;
+                    if (__any_sync(TQ_FULL_MASK, dif < 0)) {
+                        if (lane == 0) tq_status_set_thread(q, TQ_ABORTED_FULL);
+                        eok = false;
+                        break;
+                    }
+                    unsigned long long old = 0;
+                    if (lane == 0) {
+                        ++atom;
+                        old = tq_atom_cas(q.rear, pos, pos + (unsigned)p.batch);
+                        if (old != pos) ++fail;
+                    }
+                    old = tq_shfl64(old, 0);
+                    if (old == pos) {
+                        base = pos;
+                        break;
+                    }
+                }
+                et = base + lane;
+                if (active && eok) tq_st_relaxed(q.slots + (et & q.mask),
+                                                 ((unsigned long long)item << 32) | (unsigned)(et + 1));
+            }
+            if (active && eok) {
+                ++n_enq;
+                const unsigned long long f = mix64(item);
+                s_enq += f;
+                x_enq ^= f;
+                if (p.enq_log) p.enq_log[et] = item;
+            }
+            if (__any_sync(TQ_FULL_MASK, active && !eok)) break;
+
+            // ------------------------------ dequeue ------------------------------
+            uint32_t got_item = 0;
+            unsigned long long dt = 0;
+            bool have = !active;  // inactive lanes need nothing
+            if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
+                if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
+                    dt = tq_warp_dequeue_n(q, active, &atom);
+                } else if (active) {
+                    dt = tq_atom_add(q.front, 1ull);
+                    ++atom;
+                }
+                unsigned spins = 0;
+                while (!have) {
+                    have = tq_take(q, dt, &got_item);
+                    if (!have) {
+                        ++empty;
+                        if ((++spins & 1023) == 0 &&
+                            should_stop(q, (unsigned)warp_gid, deadline)) {
+                            stop = true;
+                            break;
+                        }
+                    }
+                }
+            } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
+                unsigned spins = 0;
+                while (!have) {
+                    have = b_cas_dequeue(q, &got_item, &dt, &atom, &fail);
+                    if (!have) {
+                        ++empty;
+                        if ((++spins & 1023) == 0 &&
+                            should_stop(q, (unsigned)warp_gid, deadline)) {
+                            stop = true;
+                            break;
+                        }
+                    }
+                }
+            } else {  // AN: the proxy reserves up to n ready slots per CAS
+                unsigned spins = 0;
+                for (;;) {
+                    const bool need = !have;
+                    const unsigned m = __ballot_sync(TQ_FULL_MASK, need);
+                    if (m == 0) break;
+                    const unsigned n = __popc(m);
+                    unsigned long long pos = 0;
+                    if (lane == 0) pos = tq_ld_relaxed(q.front);
+                    pos = tq_shfl64(pos, 0);
+                    int dif = -1;
+                    if (lane < n) dif = (int)((unsigned)tq_ld_relaxed(q.slots + ((pos + lane) & q.mask)) -
+                                              (unsigned)(pos + lane + 1));
+                    const unsigned rm = __ballot_sync(TQ_FULL_MASK, lane < n && dif == 0);
+                    const unsigned k = __ffs(~rm) - 1;
+                    if (k == 0) {
+                        if (!__any_sync(TQ_FULL_MASK, lane < n && dif > 0)) {
+                            if (lane == 0) ++empty;
+                            if ((++spins & 1023) == 0 &&
+                                should_stop(q, (unsigned)warp_gid, deadline)) {
+                                stop = true;
+                                break;
+                            }
+                        }
+                        continue;
+                    }
+                    unsigned long long old = 0;
+                    if (lane == 0) {
+                        ++atom;
+                        old = tq_atom_cas(q.front, pos, pos + k);
+                        if (old != pos) ++fail;
+                    }
+                    old = tq_shfl64(old, 0);
+                    if (old != pos) continue;
+                    const unsigned rank = __popc(m & tq_lanemask_lt());
+                    if (need && rank < k) {
+                        dt = pos + rank;
+                        unsigned long long *s = q.slots + (dt & q.mask);
+                        got_item = (uint32_t)(tq_ld_relaxed(s) >> 32);
+                        tq_st_relaxed(s, (unsigned long long)(unsigned)(dt + cap));
+                        have = true;
+                    }
+                }
+                stop = __any_sync(TQ_FULL_MASK, stop);
+            }
+            if (active && have) {
+                ++n_deq;
+                const unsigned long long f = mix64(got_item);
+                s_deq += f;
+                x_deq ^= f;
+                if (p.deq_log) p.deq_log[dt] = got_item;
+                uint32_t x = got_item;
+                for (int w = 0; w < p.work_iters; ++w) x = x * 1664525u + 1013904223u;
+                sink += x;
+            }
+            stop = __any_sync(TQ_FULL_MASK, stop);
+        }
+    }
+
+    // reduce and publish
+    unsigned long long v[BO_COUNT_] = {n_enq, n_deq, atom, fail, empty, s_enq, s_deq, 0, 0, sink};
+#pragma unroll
+    for (int k = 0; k < BO_COUNT_; ++k) {
+        if (k == BO_XOR_ENQ || k == BO_XOR_DEQ) continue;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v[k] += __shfl_xor_sync(TQ_FULL_MASK, v[k], o);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        x_enq ^= __shfl_xor_sync(TQ_FULL_MASK, x_enq, o);
+        x_deq ^= __shfl_xor_sync(TQ_FULL_MASK, x_deq, o);
+    }
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < BO_COUNT_; ++k) {
+            if (k == BO_XOR_ENQ || k == BO_XOR_DEQ) continue;
+            if (v[k]) atomicAdd(p.out + k, v[k]);
+        }
+        atomicXor(p.out + BO_XOR_ENQ, x_enq);
+        atomicXor(p.out + BO_XOR_DEQ, x_deq);
+    }
+}
+
+template <int V>
+static cudaError_t launch_b(const BenchParams &p, int blocks, int block, cudaStream_t s)
+{
+    bench_kernel<V><<<blocks, block, 0, s>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int block, cudaStream_t s)
+{
+    switch (variant) {
+    case TQ_VARIANT_RF_AN: return launch_b<TQ_VARIANT_RF_AN>(p, blocks, block, s);
+    case TQ_VARIANT_PER_THREAD_AFA: return launch_b<TQ_VARIANT_PER_THREAD_AFA>(p, blocks, block, s);
+    case TQ_VARIANT_CAS_RETRY: return launch_b<TQ_VARIANT_CAS_RETRY>(p, blocks, block, s);
+    case TQ_VARIANT_AN: return launch_b<TQ_VARIANT_AN>(p, blocks, block, s);
+    case TQ_VARIANT_ATOMIC_CEILING: return launch_b<TQ_VARIANT_ATOMIC_CEILING>(p, blocks, block, s);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm)
+{
+    switch (variant) {
+    case TQ_VARIANT_RF_AN:
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_RF_AN>, block, 0);
+    case TQ_VARIANT_PER_THREAD_AFA:
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_PER_THREAD_AFA>, block, 0);
+    case TQ_VARIANT_CAS_RETRY:
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_CAS_RETRY>, block, 0);
+    case TQ_VARIANT_AN:
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_AN>, block, 0);
+    case TQ_VARIANT_ATOMIC_CEILING:
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_ATOMIC_CEILING>, block, 0);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+}  // namespace tqk

@@ -1,0 +1,75 @@
+// internal.cuh -- declarations shared by the kernels (bfs.cu, bench.cu) and
+// the C-ABI implementation (api.cu).  Not part of the public boundary.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/tq.h"
+#include "../../include/tq_device.cuh"
+
+namespace tqk {
+
+// Token encoding: a 32-bit item is either a vertex
+// id (< 2^31) or CHUNK_FLAG | chunk id.  A chunk token names up to `chunk`
+// consecutive CSR entries of one high-degree vertex: the paper's refactoring
+// of a task into "a fixed number of uniformly complex sub-tasks".
+constexpr uint32_t CHUNK_FLAG = 0x80000000u;
+
+constexpr int kStatCount = 16;
+enum StatIndex {
+    ST_TASKS = 0,
+    ST_CHUNK_TASKS,
+    ST_EDGES,
+    ST_MIN_ATOMICS,
+    ST_REENQUEUES,
+    ST_QUEUE_ATOMICS,
+    ST_CAS_FAILURES,
+    ST_EMPTY_POLLS,
+    // filled by the unpack kernel
+    ST_REACHED,
+    ST_DEG_SUM,
+    ST_MAX_LEVEL,
+    ST_COUNT_
+};
+
+struct BfsParams {
+    tq_device_view q;
+    const int64_t *row_ptr;
+    const int32_t *col;
+    unsigned long long *W;     // packed (level << 32) | parent, ~0 = unreached
+    const int2 *chunk_tab;     // chunk id -> {vertex, k}
+    const int32_t *hub_base;   // vertex -> first chunk id (read for hubs only)
+    unsigned long long *stats; // kStatCount counters
+    int64_t n_vertices;
+    int chunk;                 // max edges per token (power of 2)
+    int backoff_ns;            // max idle back-off, 0 = none
+    unsigned long long timeout_ns;
+};
+
+// bfs.cu
+cudaError_t launch_bfs_init(const BfsParams &p, int32_t root, unsigned long long t0, cudaStream_t s);
+cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
+                                  cudaStream_t s);
+cudaError_t launch_bfs_unpack(const BfsParams &p, int32_t *level, int32_t *parent, cudaStream_t s);
+cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm);
+cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int32_t *hub_base,
+                              int2 **chunk_tab_out, int64_t *n_chunks_out, cudaStream_t s);
+cudaError_t launch_queue_reset(const tq_device_view &q, cudaStream_t s);
+
+// bench.cu
+struct BenchParams {
+    tq_device_view q;
+    int batch;
+    int iters;                 // per warp
+    int work_iters;
+    uint32_t seed32;
+    uint32_t *enq_log;
+    uint32_t *deq_log;
+    unsigned long long *out;   // [0..] counters (see bench.cu)
+    unsigned long long timeout_ns;
+};
+cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int block, cudaStream_t s);
+cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm);
+
+}  // namespace tqk

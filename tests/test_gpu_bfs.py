@@ -1,0 +1,193 @@
+"""GPU parity of the persistent-thread BFS (libtq, through the C ABI) against
+the sequential oracle.
+
+Levels must be identical element by element; parents must be identical under
+the min-id rule (R5) and validate Graph500-style. Every queue
+variant runs the same BFS (RF/AN, per-thread AFA, CAS-retry BASE, AN).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from inputs import (edges_to_csr, grid_csr, kronecker_csr, sample_roots, tree4_csr)
+
+pytestmark = pytest.mark.gpu
+
+VARIANTS = ["rf_an", "per_thread_afa", "cas_retry", "an"]
+
+
+@pytest.fixture(scope="module")
+def tq():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_icpp_troendletj19_b200 as m
+    return m
+
+
+def to_dev(g):
+    import torch
+    return torch.from_numpy(g.row_ptr).cuda(), torch.from_numpy(g.col).cuda()
+
+
+def check_against_oracle(g, root, level, parent, stats=None):
+    lv_o, pa_o, info = oracle.bfs(g.row_ptr, g.col, root)
+    lv = level.cpu().numpy() if hasattr(level, "cpu") else level
+    pa = parent.cpu().numpy() if hasattr(parent, "cpu") else parent
+    bad = np.flatnonzero(lv != lv_o)
+    assert bad.size == 0, f"{bad.size} level mismatches, first v={bad[0]} gpu={lv[bad[0]]} oracle={lv_o[bad[0]]}"
+    bad = np.flatnonzero(pa != pa_o)
+    assert bad.size == 0, f"{bad.size} parent mismatches, first v={bad[0]} gpu={pa[bad[0]]} oracle={pa_o[bad[0]]}"
+    assert oracle.validate_tree(g.row_ptr, g.col, root, lv, pa) == (0, -1)
+    if stats is not None:
+        assert stats["traversed_edges"] == info["traversed_edges"]
+        assert stats["reached"] == info["reached"]
+        assert stats["max_level"] == int(lv_o.max())
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_rmat10_config1_sample_roots(tq, variant):
+    g = kronecker_csr(10, 16, 1)
+    rp, col = to_dev(g)
+    import torch
+    level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+    parent = torch.empty_like(level)
+    with tq.BfsPlan(rp, col, variant=variant, timeout_s=20) as plan:
+        for root in sample_roots(g.row_ptr, 16, 2):
+            st = plan.run(int(root), level, parent)
+            check_against_oracle(g, int(root), level, parent, st)
+
+
+def test_rmat10_all_roots_rf_an(tq):
+    """Every vertex of the config-1 graph as the root, isolated ones included."""
+    import torch
+    g = kronecker_csr(10, 16, 1)
+    rp, col = to_dev(g)
+    level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+    parent = torch.empty_like(level)
+    with tq.BfsPlan(rp, col, timeout_s=20) as plan:
+        for root in range(g.n_vertices):
+            plan.run(root, level, parent)
+            check_against_oracle(g, root, level, parent)
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_small_closed_form_graphs(tq, variant):
+    graphs = [
+        edges_to_csr(np.arange(99), np.arange(1, 100), 100, "path100"),
+        edges_to_csr(np.zeros(999, dtype=np.int64), np.arange(1, 1000), 1000, "star1000"),
+        grid_csr(64, 33),
+        tree4_csr(5000),
+        edges_to_csr(np.array([0]), np.array([1]), 2, "edge"),
+        edges_to_csr(np.array([0, 0, 1, 2, 3]), np.array([1, 2, 3, 4, 4]), 8, "with_isolated"),
+    ]
+    for g in graphs:
+        rp, col = to_dev(g)
+        for root in {0, g.n_vertices // 2, g.n_vertices - 1}:
+            level, parent, st = tq.bfs(rp, col, root, variant=variant, timeout_s=20)
+            check_against_oracle(g, root, level, parent, st)
+
+
+def test_single_vertex_and_isolated_root(tq):
+    g = edges_to_csr(np.array([], dtype=np.int64), np.array([], dtype=np.int64), 1, "one")
+    rp, col = to_dev(g)
+    level, parent, st = tq.bfs(rp, col, 0)
+    assert level.tolist() == [0] and parent.tolist() == [0] and st["traversed_edges"] == 0
+    g = kronecker_csr(10, 16, 1)
+    iso = int(np.flatnonzero(g.degrees() == 0)[0])
+    rp, col = to_dev(g)
+    level, parent, st = tq.bfs(rp, col, iso)
+    check_against_oracle(g, iso, level, parent, st)
+    assert st["reached"] == 1
+
+
+def test_label_correcting_motif(tq):
+    """r-a, r-b, a-c, c-x, b-x: x has level 2 via b, not 3 via a-c (R4).
+    Repeated many times so that different schedules occur."""
+    # plus a long path hanging off a to slow one side down
+    n = 6 + 200
+    src = [0, 0, 1, 3, 2] + [1] + list(range(6, n - 1))
+    dst = [1, 2, 3, 4, 4] + [6] + list(range(7, n))
+    g = edges_to_csr(np.array(src), np.array(dst), n)
+    rp, col = to_dev(g)
+    for _ in range(20):
+        level, parent, st = tq.bfs(rp, col, 0)
+        check_against_oracle(g, 0, level, parent, st)
+
+
+@pytest.mark.parametrize("chunk", [32, 64, 1024])
+def test_hub_chunking(tq, chunk):
+    """Vertices with more than `chunk` edges are split into chunk tokens."""
+    g = kronecker_csr(14, 16, 5)
+    rp, col = to_dev(g)
+    deg = g.degrees()
+    for root in (int(np.argmax(deg)), int(sample_roots(g.row_ptr, 1, 9)[0])):
+        level, parent, st = tq.bfs(rp, col, root, chunk=chunk)
+        check_against_oracle(g, root, level, parent, st)
+        n_hub_reached = int(((deg > chunk) & (level.cpu().numpy() >= 0)).sum())
+        if n_hub_reached:
+            assert st["chunk_tasks"] > 0
+
+
+def test_host_pointers_match_device(tq):
+    g = kronecker_csr(12, 16, 3)
+    root = int(sample_roots(g.row_ptr, 1, 4)[0])
+    lh, ph, sth = tq.bfs(g.row_ptr, g.col, root)  # numpy in, numpy out
+    assert isinstance(lh, np.ndarray)
+    check_against_oracle(g, root, lh, ph, sth)
+
+
+def test_queue_full_aborts_and_retry_succeeds(tq):
+    """queue-full aborts (no retry); the user may retry with a larger queue."""
+    g = kronecker_csr(12, 16, 1)
+    rp, col = to_dev(g)
+    root = int(np.argmax(g.degrees()))
+    with pytest.raises(tq.TQError) as ei:
+        tq.bfs(rp, col, root, capacity=64)
+    assert ei.value.status == -4
+    level, parent, st = tq.bfs(rp, col, root, capacity=1 << 14)
+    check_against_oracle(g, root, level, parent, st)
+
+
+def test_plan_reuse_after_abort_and_many_runs(tq):
+    import torch
+    from inputs import kronecker_edges
+    s, d = kronecker_edges(11, 16, 2)
+    # the Kronecker graph plus a separate 300-vertex path component
+    n0 = 1 << 11
+    ps = np.arange(n0, n0 + 299, dtype=np.uint64)
+    g = edges_to_csr(np.concatenate([s, ps]), np.concatenate([d, ps + np.uint64(1)]), n0 + 300)
+    rp, col = to_dev(g)
+    level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+    parent = torch.empty_like(level)
+    roots = sample_roots(g.row_ptr[: n0 + 1], 8, 1)
+    with tq.BfsPlan(rp, col, capacity=128) as small:
+        with pytest.raises(tq.TQError) as ei:
+            small.run(int(np.argmax(g.degrees())), level, parent)
+        assert ei.value.status == -4
+        # the dirty plan resets its queue; the small component still fits
+        for _ in range(3):
+            small.run(n0 + 150, level, parent)
+            check_against_oracle(g, n0 + 150, level, parent)
+    with tq.BfsPlan(rp, col) as plan:
+        for _ in range(3):
+            for r in roots:  # tickets continue across runs without an O(C) reset
+                plan.run(int(r), level, parent)
+                check_against_oracle(g, int(r), level, parent)
+
+
+@pytest.mark.parametrize("threads", [256, 2048, 32768])
+def test_thread_counts(tq, threads):
+    g = kronecker_csr(12, 16, 7)
+    rp, col = to_dev(g)
+    root = int(sample_roots(g.row_ptr, 1, 3)[0])
+    level, parent, st = tq.bfs(rp, col, root, threads=threads)
+    check_against_oracle(g, root, level, parent, st)
+    assert st["persistent_threads"] == threads
+
+
+def test_no_backoff_and_large_backoff(tq):
+    g = grid_csr(128, 128)
+    rp, col = to_dev(g)
+    for b in (-1, 4096):
+        level, parent, st = tq.bfs(rp, col, 0, backoff_ns=b)
+        check_against_oracle(g, 0, level, parent, st)
