@@ -1,0 +1,381 @@
+#!/usr/bin/env python
+"""Benchmark: batched multi-root persistent-thread BFS on the retry-free,
+arbitrary-n queue (BASELINE.json configs[4]: Kronecker scale 26, edgefactor
+16, 64 roots split across the ranks, graph replicated, NCCL stats gather).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tq|reference]
+                    [--workload kron26x64|kron24x64|kron24x8|grid4096|rmat10]
+
+A step is one pass of the whole hot path over one batch: for every root of
+this rank's share, queue/state init (a2) + persistent BFS (a3-a8) + unpack
+and stats (a9). The metric is GTEPS = sum over roots of traversed edges
+(undirected, deduplicated, loop-free edges with a reached endpoint; DESIGN.md
+R16) / the step time (max over ranks). Rank 0 prints ONE JSON line.
+
+--impl reference runs the oracle (oracle/, the plain sequential C BFS) on the
+host cores, on a bounded sample of the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (kind, scale/rows, edgefactor, n_roots)
+    "kron26x64": ("kron", 26, 16, 64),
+    "kron24x64": ("kron", 24, 16, 64),
+    "kron24x8": ("kron", 24, 16, 8),
+    "grid4096": ("grid", 4096, 0, 1),
+    "rmat10": ("kron", 10, 16, 16),
+}
+GRAPH_SEED, ROOT_SEED = 1, 2
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi-equivalent clock / throttle sampling (NVML) during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+        0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+        0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+    }
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            self._stop.wait(0.1)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        s = sorted(self.samples)
+        return {"sm_mhz": s[len(s) // 2] if s else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(s)}
+
+
+def make_graph(kind, a, ef, device):
+    import inputs.gpu as gg
+    gg.build()
+    if kind == "kron":
+        return gg.kronecker_csr_cuda(a, ef, GRAPH_SEED, device=device)
+    return gg.grid_csr_cuda(a, a, device=device)
+
+
+def pick_roots(kind, row_ptr_host, n_roots):
+    from inputs import sample_roots
+    if kind == "grid":
+        return [0]  # corner: 8,191 levels (R17)
+    return [int(r) for r in sample_roots(row_ptr_host, n_roots, ROOT_SEED)]
+
+
+def algorithmic_bytes(traversed_edges, reached):
+    """SURVEY §8(d) per-unit figures for the persistent kernel (DESIGN.md
+    "Algorithmic bytes"): 12 B per directed CSR entry of a reached vertex
+    (4 B col + 8 B W prefilter) and 56 B per reached vertex (16 B row_ptr,
+    24 B queue slot write/poll/reset, 8 B W install, 8 B fresh level read)."""
+    return 12 * 2 * traversed_edges + 56 * reached
+
+
+def cpu_oracle_sample(row_ptr, col, roots, budget_s=20.0, check=None):
+    """Time the oracle (as it stands, 1 core) on roots of the same graph until
+    the budget is spent; returns (teps, sample description, levels of root 0)."""
+    import oracle
+    te_sum, sec_sum, done, lv0 = 0, 0.0, [], None
+    for r in roots:
+        lv, _, info = oracle.bfs(row_ptr, col, r, parents=False)
+        te_sum += info["traversed_edges"]
+        sec_sum += info["seconds_levels"]
+        done.append(r)
+        if lv0 is None:
+            lv0 = lv
+        if sec_sum >= budget_s:
+            break
+    return te_sum / sec_sum, done, sec_sum, lv0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="tq", choices=["tq", "reference"])
+    ap.add_argument("--workload", default=os.environ.get("TQ_BENCH_WORKLOAD", "kron26x64"),
+                    choices=sorted(WORKLOADS))
+    ap.add_argument("--variant", default="rf_an")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=20.0)
+    args = ap.parse_args()
+
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    kind, a, ef, n_roots = WORKLOADS[args.workload]
+    hbm_peak, peak_src = peaks()
+
+    import numpy as np
+    import torch
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        run_reference(args, kind, a, ef, n_roots)
+        return
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+
+    import paper_conf_icpp_troendletj19_b200 as tq
+
+    # ---- inputs (not timed): generated on the device, replicated per rank ----
+    t_gen = time.time()
+    row_ptr, col = make_graph(kind, a, ef, dev)
+    rp_host = row_ptr.cpu().numpy()
+    roots = pick_roots(kind, rp_host, n_roots)
+    mine = roots[rank * len(roots) // world:(rank + 1) * len(roots) // world]
+    n = int(row_ptr.numel()) - 1
+    t_gen = time.time() - t_gen
+
+    stream = torch.cuda.current_stream(dev)
+    plan = tq.BfsPlan(row_ptr, col, variant=args.variant, stream=stream, device=local)
+    level = torch.empty(n, dtype=torch.int32, device=dev)
+    parent = torch.empty(n, dtype=torch.int32, device=dev)
+
+    def step():
+        sts = []
+        for r in mine:
+            sts.append(plan.run(r, level, parent))
+        return sts
+
+    for _ in range(args.warmup):
+        step()
+
+    # ---- timed region: K steps, barrier + sync on both sides, device events ----
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    all_stats = []
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            all_stats.extend(step())
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+    if dist:
+        dist.barrier()
+    ms_total = e0.elapsed_time(e1)
+    te_local = sum(s["traversed_edges"] for s in all_stats)
+    reached_local = sum(s["reached"] for s in all_stats)
+    kern_ms_local = sum(s["ms_kernel"] for s in all_stats)
+    launches_local = 3 * len(all_stats)
+
+    # NCCL gather of per-rank stats (the only collective; outside the data path)
+    vec = torch.tensor([ms_total, te_local, reached_local, kern_ms_local, launches_local,
+                        len(all_stats)], dtype=torch.float64, device=dev)
+    if dist:
+        out = torch.empty(world * vec.numel(), dtype=torch.float64, device=dev)
+        dist.all_gather_into_tensor(out, vec)
+        allv = out.view(world, -1).cpu().numpy()
+    else:
+        allv = vec.view(1, -1).cpu().numpy()
+    ms_max = float(allv[:, 0].max())
+    te_all = float(allv[:, 1].sum())
+    reached_all = float(allv[:, 2].sum())
+    kern_ms_all = float(allv[:, 3].sum())
+    launches = int(allv[:, 4].sum())
+    runs_all = int(allv[:, 5].sum())
+
+    gteps = te_all / (ms_max * 1e-3) / 1e9
+    ms_per_step = ms_max / args.steps
+
+    # roofline of the dominant kernel (bfs_persistent), per launch
+    alg_bytes = algorithmic_bytes(te_all, reached_all) / runs_all
+    avg_kernel_s = kern_ms_all / runs_all * 1e-3
+    achieved = alg_bytes / avg_kernel_s / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+
+    # ---- e2e through the public API with host buffers (pinned), every step ----
+    e2e = None
+    if not args.no_e2e:
+        rp_pin = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
+        col_pin = torch.empty(col.numel(), dtype=torch.int32, pin_memory=True)
+        rp_pin.copy_(row_ptr)
+        col_pin.copy_(col)
+        lv_pin = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        pa_pin = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        rp_np, col_np, lv_np, pa_np = rp_pin.numpy(), col_pin.numpy(), lv_pin.numpy(), pa_pin.numpy()
+        del plan
+        torch.cuda.empty_cache()
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        te_e2e = 0
+        for _ in range(args.steps):
+            with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=stream, device=local) as hp:
+                for r in mine:
+                    s = hp.run(r, lv_np, pa_np)
+                    te_e2e += s["traversed_edges"]
+        torch.cuda.synchronize(dev)
+        sec = time.perf_counter() - t0
+        secv = torch.tensor([sec, te_e2e], dtype=torch.float64, device=dev)
+        if dist:
+            o2 = torch.empty(world * 2, dtype=torch.float64, device=dev)
+            dist.all_gather_into_tensor(o2, secv)
+            o2 = o2.view(world, 2).cpu().numpy()
+            sec_max, te_tot = float(o2[:, 0].max()), float(o2[:, 1].sum())
+        else:
+            sec_max, te_tot = sec, float(te_e2e)
+        e2e = {"value": te_tot / sec_max / 1e9, "unit": "GTEPS",
+               "h2d_bytes_per_step": int((n + 1) * 8 + col.numel() * 4),
+               "d2h_bytes_per_step": int(len(mine) * n * 8),
+               "timed": "host perf_counter around plan_create(host CSR) + run(host outputs) per root, synchronised"}
+
+    # ---- CPU baseline: the oracle, 1 core, bounded sample, rank 0 at N=1 ----
+    cpu = None
+    parity = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        col_host = col.cpu().numpy()
+        teps, done, sec, lv0 = cpu_oracle_sample(rp_host, col_host, mine, args.cpu_budget)
+        plan2 = tq.BfsPlan(row_ptr, col, variant=args.variant, device=local)
+        plan2.run(done[0], level, parent)
+        parity = bool(np.array_equal(level.cpu().numpy(), lv0))
+        plan2.close()
+        cpu = {"value": teps / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+               "sample": f"{len(done)} of the {len(roots)} roots of the same graph, sequential "
+                         f"BFS levels only ({sec:.1f} s of CPU)"}
+
+    if rank == 0:
+        line = {
+            "metric": "BFS GTEPS (batched multi-root, persistent-thread RF/AN queue)",
+            "value": round(gteps, 4),
+            "unit": "GTEPS",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": round(ms_per_step, 3),
+            "higher_is_better": True,
+            "scaling": "strong",
+            "vs_baseline": None,
+            "dtype": "int32/int64 (integer path)",
+            "data": "synthetic (seeded Kronecker/Graph500 R-MAT generated on the device)",
+            "config": {"workload": args.workload, "graph": f"{kind} {a}" + (f" ef{ef}" if ef else ""),
+                       "n_vertices": n, "nnz": int(col.numel()), "roots_total": len(roots),
+                       "roots_per_rank": len(mine), "variant": args.variant,
+                       "parallelism": f"roots split over {world} rank(s), graph replicated",
+                       "l2": "inputs larger than L2 (CSR >> 126 MB)",
+                       "persistent_threads": all_stats[0]["persistent_threads"]},
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak,
+                         "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": traffic,
+                         "kernel": "bfs_persistent_kernel<RF_AN>", "peak_source": peak_src,
+                         "alg_bytes_per_launch": int(alg_bytes),
+                         "avg_launch_ms": round(avg_kernel_s * 1e3, 4)},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+            "parity_sampled_root_levels_identical": parity,
+            "graph_gen_s": round(t_gen, 2),
+        }
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+def run_reference(args, kind, a, ef, n_roots):
+    """--impl reference: the oracle as it stands on the host cores."""
+    import numpy as np
+    import torch
+
+    import oracle
+    dev = torch.device("cuda", 0) if torch.cuda.is_available() else None
+    if dev is not None:
+        row_ptr, col = make_graph(kind, a, ef, dev)
+        rp, cl = row_ptr.cpu().numpy(), col.cpu().numpy()
+        del row_ptr, col
+    else:  # CPU-only host: numpy generator (small workloads only)
+        from inputs import grid_csr, kronecker_csr
+        g = kronecker_csr(a, ef, GRAPH_SEED) if kind == "kron" else grid_csr(a)
+        rp, cl = g.row_ptr, g.col
+    roots = pick_roots(kind, rp, n_roots)
+    oracle.build()
+
+    def step(i):
+        r = roots[i % len(roots)]
+        _, _, info = oracle.bfs(rp, cl, r, parents=False)
+        return info["traversed_edges"], info["seconds_levels"]
+
+    for i in range(args.warmup):
+        step(i)
+    te, sec = 0, 0.0
+    for i in range(args.steps):
+        t, s = step(args.warmup + i)
+        te += t
+        sec += s
+    v = te / sec / 1e9
+    print(json.dumps({
+        "impl": "reference", "metric": "BFS GTEPS (batched multi-root, persistent-thread RF/AN queue)",
+        "value": round(v, 6), "unit": "GTEPS", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(sec / args.steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "int32/int64 (integer path)", "data": "synthetic",
+        "config": {"workload": args.workload},
+        "cpu_baseline": {"value": round(v, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                         "sample": f"one root of the workload per step ({args.steps} steps)"},
+        "e2e": {"value": round(v, 6), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+if __name__ == "__main__":
+    main()

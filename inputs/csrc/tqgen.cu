@@ -191,6 +191,7 @@ int tqgen_sort_unique(uint64_t *keys, uint64_t *alt, int64_t n, int64_t *n_out, 
     int64_t *d_count = nullptr;
     e = e == cudaSuccess ? cub::DeviceSelect::Unique(nullptr, tmp2, keys, alt, d_count, n, stream) : e;
     if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
+    tmp_bytes = (tmp_bytes + 255) & ~(size_t)255;  // d_count follows, 8-byte aligned
     void *tmp = nullptr;
     if (e == cudaSuccess) e = cudaMalloc(&tmp, tmp_bytes + 256);
     if (e == cudaSuccess) {

@@ -44,7 +44,7 @@ __device__ __forceinline__ bool bench_publish(const tq_device_view &q, unsigned 
 __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t item,
                                               unsigned long long *t_out, unsigned *atom, unsigned *fail)
 {
-    for (;;) {
+    for (unsigned tries = 0; tries < (1u << 24); ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.rear);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -62,12 +62,14 @@ __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t 
             return false;
         }
     }
+    tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
+    return false;
 }
 
 __device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *item,
                                              unsigned long long *t_out, unsigned *atom, unsigned *fail)
 {
-    for (;;) {
+    for (unsigned tries = 0; tries < (1u << 12); ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.front);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -85,6 +87,7 @@ __device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *
             return 0;
         }
     }
+    return 0;
 }
 
 // polled every 1024 empty spins: watchdog + abort propagation
@@ -139,8 +142,12 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                 if (active) eok = b_cas_enqueue(q, item, &et, &atom, &fail);
             } else {  // AN: proxy CAS loop reserving `batch` slots
                 unsigned long long base = 0;
-                // reuse the BFS AN reservation logic inline
+                unsigned spins = 0;
                 for (;;) {
+                    if ((++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {
+                        eok = false;
+                        break;
+                    }
                     unsigned long long pos = 0;
                     if (lane == 0) pos = tq_ld_relaxed(q.rear);
                     pos = tq_shfl64(pos, 0);
@@ -220,6 +227,10 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                     const bool need = !have;
                     const unsigned m = __ballot_sync(TQ_FULL_MASK, need);
                     if (m == 0) break;
+                    if ((++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {
+                        stop = true;
+                        break;
+                    }
                     const unsigned n = __popc(m);
                     unsigned long long pos = 0;
                     if (lane == 0) pos = tq_ld_relaxed(q.front);
@@ -228,16 +239,9 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                     if (lane < n) dif = (int)((unsigned)tq_ld_relaxed(q.slots + ((pos + lane) & q.mask)) -
                                               (unsigned)(pos + lane + 1));
                     const unsigned rm = __ballot_sync(TQ_FULL_MASK, lane < n && dif == 0);
-                    const unsigned k = __ffs(~rm) - 1;
+                    const unsigned k = rm == TQ_FULL_MASK ? 32u : (unsigned)(__ffs(~rm) - 1);
                     if (k == 0) {
-                        if (!__any_sync(TQ_FULL_MASK, lane < n && dif > 0)) {
-                            if (lane == 0) ++empty;
-                            if ((++spins & 1023) == 0 &&
-                                should_stop(q, (unsigned)warp_gid, deadline)) {
-                                stop = true;
-                                break;
-                            }
-                        }
+                        if (!__any_sync(TQ_FULL_MASK, lane < n && dif > 0) && lane == 0) ++empty;
                         continue;
                     }
                     unsigned long long old = 0;

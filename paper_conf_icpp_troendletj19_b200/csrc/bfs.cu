@@ -34,6 +34,11 @@ constexpr int kBlock = 256;          // threads per block (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr int kStageCap = 512;       // staged tokens per warp (2 KiB smem)
 constexpr int kU = 4;                // 32-edge rounds in flight per lane
+// bound on CAS retries of one operation; reaching it can only mean a broken
+// queue state (the loops are lock-free), which is reported as a timeout
+constexpr unsigned kMaxEnqRetries = 1u << 24;
+// a dequeue that keeps losing simply reports "empty" and retries next cycle
+constexpr unsigned kMaxDeqRetries = 1u << 12;
 
 __device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long *p)
 {
@@ -93,7 +98,7 @@ __device__ __forceinline__ T warp_sum(T x)
 __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_t *item,
                                                 unsigned *atom, unsigned *fail)
 {
-    for (;;) {
+    for (unsigned tries = 0; tries < kMaxDeqRetries; ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.front);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -110,13 +115,14 @@ __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_
             return false;  // queue empty: the exception BASE retries on
         }
     }
+    return false;
 }
 
 // BASE enqueue of one item by one lane; queue-full aborts (no retry).
 __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_t item,
                                                 unsigned *atom, unsigned *fail)
 {
-    for (;;) {
+    for (unsigned tries = 0; tries < kMaxEnqRetries; ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.rear);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -133,6 +139,8 @@ __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_
             return false;
         }
     }
+    tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
+    return false;
 }
 
 // AN dequeue: the proxy reserves up to n ready slots with one CAS (retrying on
@@ -143,6 +151,7 @@ __device__ __forceinline__ unsigned an_dequeue(const tq_device_view &q, unsigned
                                                unsigned *fail)
 {
     const unsigned lane = tq_lane();
+    unsigned tries = 0;
     for (;;) {
         unsigned long long pos = 0;
         if (lane == 0) pos = tq_ld_relaxed(q.front);
@@ -155,11 +164,11 @@ __device__ __forceinline__ unsigned an_dequeue(const tq_device_view &q, unsigned
             ready = dif == 0;
         }
         const unsigned rm = __ballot_sync(TQ_FULL_MASK, ready);
-        const unsigned k = __ffs(~rm) - 1;  // leading ready slots
+        const unsigned k = rm == TQ_FULL_MASK ? 32u : (unsigned)(__ffs(~rm) - 1);  // leading ready slots
         const unsigned stale = __ballot_sync(TQ_FULL_MASK, lane < n && dif > 0);
         if (k == 0) {
-            if (stale & 1u) continue;  // Front moved on under us: retry
-            return 0;                  // empty
+            if ((stale & 1u) && ++tries < kMaxDeqRetries) continue;  // Front moved on: retry
+            return 0;                                             // empty
         }
         unsigned long long old = 0;
         if (lane == 0) {
@@ -172,6 +181,7 @@ __device__ __forceinline__ unsigned an_dequeue(const tq_device_view &q, unsigned
             *base_out = pos;
             return k;
         }
+        if (++tries >= kMaxDeqRetries) return 0;
     }
 }
 
@@ -182,7 +192,11 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
                                                 unsigned *fail)
 {
     const unsigned lane = tq_lane();
-    for (;;) {
+    for (unsigned tries = 0;; ++tries) {
+        if (tries >= kMaxEnqRetries) {
+            if (lane == 0) tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
+            return false;
+        }
         unsigned long long pos = 0;
         if (lane == 0) pos = tq_ld_relaxed(q.rear);
         pos = tq_shfl64(pos, 0);

@@ -24,7 +24,8 @@ def tq():
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("warps,batch", [(1, 1), (1, 32), (7, 5), (64, 32), (0, 8)])
 def test_conservation(tq, variant, warps, batch):
-    r = tq.queue_bench(variant, warps=warps, batch=batch, items=1 << 16, capacity=1 << 14,
+    items = 1 << 16 if warps else 1 << 22  # full occupancy needs >= 1 item per lane
+    r = tq.queue_bench(variant, warps=warps, batch=batch, items=items, capacity=1 << 20,
                        seed=11, timeout_s=30)
     exp = fingerprint(item_of(11, np.arange(r["items"])))
     assert (r["enq"], r["sum_enq"], r["xor_enq"]) == exp
