@@ -145,7 +145,14 @@ typedef struct {
                            < 0 = none                                        */
     int device;         /* CUDA device for bfs_plan_create / host-pointer runs;
                            ignored when the CSR is device memory             */
+    int parent_rule;    /* TQ_PARENT_ANY (0, default): some neighbour one level
+                           up (a valid Graph500 BFS tree; schedule-dependent);
+                           TQ_PARENT_MIN_ID (1): the smallest-id neighbour one
+                           level up (unique, bit-exact; ~20% slower: level
+                           ties must consult the packed word)               */
 } bfs_opts;
+
+enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };
 
 /* Per-run statistics (device counters, summed over warps). */
 typedef struct {
@@ -162,13 +169,16 @@ typedef struct {
     uint64_t cas_failures;      /* CAS variants only                           */
     uint64_t empty_polls;       /* work cycles that found no data              */
     uint64_t tickets;           /* tasks enqueued (Rear advance)               */
+    uint64_t skipped_tasks;     /* vertex tokens dropped by the expanded-level
+                                   marker (already expanded at <= level)      */
     int32_t max_level;
     int32_t persistent_threads;
 } bfs_stats;
 
 /* Single-source BFS.  level_out[v] = hop distance from root (-1 unreached);
- * parent_out[v] = the smallest-id neighbour one level closer to the root
- * (parent_out[root] = root, -1 unreached).  Either output may be NULL.
+ * parent_out[v] = a neighbour one level closer to the root (the smallest-id
+ * one under TQ_PARENT_MIN_ID), parent_out[root] = root, -1 unreached.
+ * Either output may be NULL.
  * Graph and outputs: host or device pointers (device pointers must be on the
  * current device).  Synchronous.  Returns TQ_ERR_QUEUE_FULL if the queue
  * overflowed (retry with a larger opts->capacity). */

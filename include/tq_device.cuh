@@ -47,6 +47,17 @@ __device__ __forceinline__ unsigned int tq_ld_relaxed_u32(const unsigned int *p)
     asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ unsigned long long tq_ld_acquire(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+/* fire-and-forget add with release semantics (completion counter) */
+__device__ __forceinline__ void tq_red_add_release(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void tq_st_relaxed(unsigned long long *p, unsigned long long v)
 {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -158,6 +169,19 @@ __device__ __forceinline__ unsigned long long tq_warp_dequeue_n(const tq_device_
 /* next lap ("picks up its work token from its slot and replaces it   */
 /* with the sentinel").  Non-blocking; per lane.               */
 /* ---------------------------------------------------------------- */
+/* The arrival check alone (Listing 2 lines 3-5): true if the item for
+ * `ticket` has arrived.  The caller takes it: tq_fence_gpu() (acquire), then
+ * stores seq = ticket + C to the slot (the reset half of tq_take). */
+__device__ __forceinline__ bool tq_poll(const tq_device_view &q, unsigned long long ticket,
+                                        unsigned int *item)
+{
+    if (ticket == TQ_NO_TICKET) return false;
+    const unsigned long long v = tq_ld_relaxed(q.slots + (ticket & q.mask));
+    if ((unsigned int)v != (unsigned int)(ticket + 1)) return false;
+    *item = (unsigned int)(v >> 32);
+    return true;
+}
+
 __device__ __forceinline__ bool tq_take(const tq_device_view &q, unsigned long long ticket,
                                         unsigned int *item)
 {

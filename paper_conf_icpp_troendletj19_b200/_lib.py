@@ -18,6 +18,7 @@ TQ_OK, TQ_ERR_INVALID, TQ_ERR_CUDA, TQ_ERR_NOMEM, TQ_ERR_QUEUE_FULL, TQ_ERR_TIME
 
 VARIANTS = {"rf_an": 0, "per_thread_afa": 1, "cas_retry": 2, "an": 3, "atomic_ceiling": 4}
 STATUS_NAMES = {0: "running", 1: "finished", 2: "aborted_full", 3: "aborted_timeout"}
+PARENT_RULES = {"any": 0, "min_id": 1}
 
 
 class tq_device_view(ctypes.Structure):
@@ -36,7 +37,8 @@ class tq_csr(ctypes.Structure):
 class bfs_opts(ctypes.Structure):
     _fields_ = [("capacity", c_u64), ("threads", ctypes.c_int), ("block", ctypes.c_int),
                 ("chunk", ctypes.c_int), ("variant", ctypes.c_int), ("stream", c_vp),
-                ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int)]
+                ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int),
+                ("parent_rule", ctypes.c_int)]
 
 
 class bfs_stats(ctypes.Structure):
@@ -44,7 +46,7 @@ class bfs_stats(ctypes.Structure):
                 ("tasks", c_u64), ("chunk_tasks", c_u64), ("edges_scanned", c_u64),
                 ("min_atomics", c_u64), ("reenqueues", c_u64), ("queue_atomics", c_u64),
                 ("cas_failures", c_u64), ("empty_polls", c_u64), ("tickets", c_u64),
-                ("max_level", c_i32), ("persistent_threads", c_i32)]
+                ("skipped_tasks", c_u64), ("max_level", c_i32), ("persistent_threads", c_i32)]
 
 
 class tq_bench_cfg(ctypes.Structure):

@@ -97,7 +97,7 @@ struct tq_queue {
 struct bfs_plan {
     int device = 0;
     cudaStream_t stream = nullptr;
-    int variant = 0, block = 256, blocks = 0, chunk = 256, backoff_ns = 256;
+    int variant = 0, block = 256, blocks = 0, chunk = 256, backoff_ns = 256, parent_rule = 0;
     double timeout_s = 60.0;
     int64_t n = 0, nnz = 0;
     int64_t *row_ptr = nullptr;
@@ -105,6 +105,8 @@ struct bfs_plan {
     bool owns_graph = false;
     unsigned long long *W = nullptr;
     int32_t *hub_base = nullptr;
+    uint8_t *lvl8 = nullptr;
+    int32_t *xl = nullptr;
     int2 *chunk_tab = nullptr;
     int64_t n_chunks = 0;
     tq_queue *q = nullptr;
@@ -246,6 +248,8 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     }
     cudaFree(p->W);
     cudaFree(p->hub_base);
+    cudaFree(p->lvl8);
+    cudaFree(p->xl);
     cudaFree(p->chunk_tab);
     cudaFree(p->stats);
     cudaFree(p->out_scratch);
@@ -286,6 +290,11 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     p->chunk = chunk;
     p->backoff_ns = o.backoff_ns == 0 ? 256 : (o.backoff_ns < 0 ? 0 : o.backoff_ns);
     p->timeout_s = o.timeout_s > 0 ? o.timeout_s : 60.0;
+    if (o.parent_rule != TQ_PARENT_MIN_ID && o.parent_rule != TQ_PARENT_ANY) {
+        delete p;
+        return TQ_ERR_INVALID;
+    }
+    p->parent_rule = o.parent_rule;
     p->n = n;
     p->nnz = nnz;
 
@@ -311,6 +320,8 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     }
     e = cudaMalloc(&p->W, (size_t)n * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMalloc(&p->hub_base, (size_t)n * sizeof(int32_t));
+    if (e == cudaSuccess) e = cudaMalloc(&p->lvl8, (size_t)n);
+    if (e == cudaSuccess) e = cudaMalloc(&p->xl, (size_t)n * sizeof(int32_t));
     if (e == cudaSuccess) e = cudaMalloc(&p->stats, kStatCount * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
     for (auto &ev : p->ev)
@@ -358,6 +369,10 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     bp.W = p->W;
     bp.chunk_tab = p->chunk_tab;
     bp.hub_base = p->hub_base;
+    bp.lvl8 = p->lvl8;
+    bp.xl = p->xl;
+    bp.parent_rule = p->parent_rule;
+    bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;
     bp.stats = p->stats;
     bp.n_vertices = p->n;
     bp.chunk = p->chunk;
@@ -410,6 +425,7 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
         stats->traversed_edges = h[ST_DEG_SUM] / 2;
         stats->max_level = (int32_t)h[ST_MAX_LEVEL];
         stats->tickets = ctr[1] - t0;
+        stats->skipped_tasks = h[ST_SKIPPED];
         stats->persistent_threads = p->blocks * p->block;
     }
     if (status == TQ_FINISHED) return TQ_OK;

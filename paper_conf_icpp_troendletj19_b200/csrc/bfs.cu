@@ -34,6 +34,12 @@ constexpr int kBlock = 256;          // threads per block (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr int kStageCap = 512;       // staged tokens per warp (2 KiB smem)
 constexpr int kU = 4;                // 32-edge rounds in flight per lane
+// Resident blocks per SM requested from ptxas (48 warps/SM; <= 40 registers).
+// The expansion is latency-bound (long-scoreboard stalls on col / mirror /
+// atomicMin); measured on B200 kron24: 6 blocks (40 regs, ~40 B spills) beat
+// 4 blocks (64 regs) by 1.2x and 8 blocks (32 regs, more spills) by 1.07x.
+constexpr int kMinBlocks = 6;
+constexpr unsigned kLvlSat = 254;    // byte mirror: 0..253 exact, 254 = ">= 254", 255 = unreached
 // bound on CAS retries of one operation; reaching it can only mean a broken
 // queue state (the loops are lock-free), which is reported as a timeout
 constexpr unsigned kMaxEnqRetries = 1u << 24;
@@ -57,6 +63,27 @@ __device__ __forceinline__ int64_t ld_nc_i64(const int64_t *p)
     int64_t v;
     asm("ld.global.nc.s64 %0, [%1];" : "=l"(v) : "l"(p));
     return v;
+}
+
+__device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p)
+{
+    unsigned v;
+    asm volatile("ld.global.cg.u8 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ void st_u8(uint8_t *p, unsigned v)
+{
+    asm volatile("st.global.u8 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ int ld_relaxed_i32(const int32_t *p)
+{
+    int v;
+    asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_i32(int32_t *p, int v)
+{
+    asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
 // number of lanes whose inclusive prefix `incl` is <= g (owner lane of g)
@@ -233,7 +260,7 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const uint32_t *items,
                                                unsigned cnt, unsigned lane, unsigned *qatom,
-                                               unsigned *casfail)
+                                               unsigned *casfail, unsigned flags = 0)
 {
     if (cnt == 0) return;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
@@ -243,7 +270,7 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
         } else {
             if (!an_reserve_rear(q, cnt, &base, qatom, casfail)) return;
         }
-        tq_fence_gpu();  // release: W updates before the tokens that name them
+        if (!(flags & 2)) tq_fence_gpu();  // release: W updates before the tokens that name them
         for (unsigned i0 = 0; i0 < cnt; i0 += 32 * 4) {
             unsigned long long sv[4];
 #pragma unroll
@@ -315,8 +342,8 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
 // ---------------------------------------------------------------------------
 // The persistent kernel
 // ---------------------------------------------------------------------------
-template <int VARIANT>
-__global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams p)
+template <int VARIANT, int KU = kU, int MINB = kMinBlocks>
+__global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsParams p)
 {
     __shared__ uint32_t stage_all[kWarps][kStageCap];
     const unsigned lane = threadIdx.x & 31;
@@ -326,33 +353,62 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
     const unsigned long long cap = q.mask + 1;
     const int chunk = p.chunk;
 
-    unsigned long long ticket = TQ_NO_TICKET;  // the lane's DequeueThreadSlotIndex
-    unsigned st_tasks = 0, st_chunks = 0, st_min = 0, st_reenq = 0, st_qatom = 0, st_fail = 0,
-             st_empty = 0;
-    unsigned long long st_edges = 0;
-    unsigned backoff = 0, idle = 0;
-    const unsigned long long deadline = tq_globaltimer() + p.timeout_ns;
+    // The lane's DequeueThreadSlotIndex.  Only the low 32 bits of the 64-bit
+    // ticket are kept: with C <= 2^31 they fix both the slot (t & mask) and
+    // the sequence tag (u32)(t + 1) the slot protocol compares.
+    unsigned tk = 0;
+    bool have = false;
+    const unsigned cap32 = (unsigned)cap;
+    // statistics: per-warp counters in shared memory, updated by lane 0 with
+    // warp-aggregated counts (keeps them out of the hot loop's registers)
+    __shared__ unsigned long long wst_all[kWarps][kStatCount];
+    __shared__ unsigned long long wdeadline[kWarps];
+    unsigned long long *S = wst_all[threadIdx.x >> 5];
+    if (lane < kStatCount) S[lane] = 0;
+    if (lane == 0) wdeadline[threadIdx.x >> 5] = tq_globaltimer() + p.timeout_ns;
+    __syncwarp();
+    unsigned st_qatom = 0, st_fail = 0;
+    const bool min_id = p.parent_rule == TQ_PARENT_MIN_ID;
+    unsigned backoff = 0, idle = 0, busy = 0;
+
+    // Listing 1, split in two halves: the proxy's
+    // atomic_add(Front, n) for the lanes that became hungry is issued right
+    // after their take and its result is consumed one cycle later, so the
+    // atomic's latency hides behind the expansion.
+    unsigned pend_base = 0;  // lane 0: (low half of the) base of the in-flight reservation
+    unsigned pend_mask = 0;  // warp-uniform: lanes waiting for it
+    if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
+        pend_mask = TQ_FULL_MASK;
+        if (lane == 0) {
+            pend_base = (unsigned)tq_atom_add(q.front, 32ull);
+            ++st_qatom;
+        }
+    }
 
     for (;;) {
-        // ---- Algorithm 1 line 1: WorkRemains() ----
-        if (tq_status_read(q, warp_gid) != TQ_RUNNING) break;
-
         // ---- Listing 1 + Listing 2: GetWorkToken() ----
         bool got = false;
         uint32_t item = 0;
-        if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
-            const bool hungry = ticket == TQ_NO_TICKET;
-            const unsigned long long t = tq_warp_dequeue_n(q, hungry, &st_qatom);
-            if (hungry) ticket = t;
-            got = tq_take(q, ticket, &item);
-            if (got) ticket = TQ_NO_TICKET;
-        } else if constexpr (VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
-            if (ticket == TQ_NO_TICKET) {
-                ticket = tq_atom_add(q.front, 1ull);
+        if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
+            if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
+                if (pend_mask) {  // Listing 1 lines 16-19
+                    const unsigned base = __shfl_sync(TQ_FULL_MASK, pend_base, 0);
+                    if (pend_mask >> lane & 1u) {
+                        tk = base + __popc(pend_mask & tq_lanemask_lt());
+                        have = true;
+                    }
+                    pend_mask = 0;
+                }
+            } else if (!have) {
+                tk = (unsigned)tq_atom_add(q.front, 1ull);
+                have = true;
                 ++st_qatom;
             }
-            got = tq_take(q, ticket, &item);
-            if (got) ticket = TQ_NO_TICKET;
+            if (have) {  // Listing 2 lines 3-5: non-atomic arrival check
+                const unsigned long long sv = tq_ld_relaxed(q.slots + (tk & q.mask));
+                got = (unsigned)sv == tk + 1u;
+                item = (uint32_t)(sv >> 32);
+            }
         } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
             got = cas_dequeue_one(q, &item, &st_qatom, &st_fail);
         } else {  // AN: every lane is hungry each cycle (no held tickets)
@@ -368,18 +424,49 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
         }
         const unsigned gm = __ballot_sync(TQ_FULL_MASK, got);
         if (gm == 0) {
-            if (lane == 0) ++st_empty;
+            // ---- idle work cycle: Algorithm 1 line 1, WorkRemains() ----
+            if (lane == 0) ++S[ST_EMPTY_POLLS];
+            ++idle;
+            if ((idle & 3) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
+            if ((idle & 15) == 0) {
+                bool fin = false;
+                if (lane == 0) {
+                    // Done is read before Rear (R6): done(t1) ==
+                    // rear(t2), t1 < t2, implies nothing is queued or in flight
+                    const unsigned long long d = tq_ld_acquire(q.done);
+                    fin = d == tq_ld_relaxed(q.rear);
+                    if (!fin && tq_globaltimer() > wdeadline[threadIdx.x >> 5])
+                        tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
+                }
+                if (__any_sync(TQ_FULL_MASK, fin)) {
+                    tq_warp_status_set(q, TQ_FINISHED);
+                    break;
+                }
+            }
             if (p.backoff_ns > 0) {
                 backoff = backoff ? min(backoff * 2, (unsigned)p.backoff_ns) : 32u;
                 __nanosleep(backoff);
             }
-            if ((++idle & 63) == 0 && tq_globaltimer() > deadline) {
-                if (lane == 0) tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
-            }
             continue;
         }
         backoff = 0;
-        tq_fence_gpu();  // acquire: the producer's W update is visible now
+        idle = 0;
+        if (((++busy) & 63) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
+        if (!(p.exp_flags & 1)) tq_fence_gpu();  // acquire: the producer's W update is visible now
+        if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
+            if (got) {  // put the slot back to dna for the next lap
+                tq_st_relaxed(q.slots + (tk & q.mask), (unsigned long long)(tk + cap32));
+                have = false;
+            }
+        }
+        if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
+            // first half of the next dequeue (Listing 1 lines 12-14)
+            pend_mask = gm;
+            if (lane == 0) {
+                pend_base = (unsigned)tq_atom_add(q.front, (unsigned long long)__popc(gm));
+                ++st_qatom;
+            }
+        }
 
         // ---- enumeration prolog (Listing 2 lines 6-22) ----
         int32_t v = 0;
@@ -387,10 +474,9 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
         unsigned nch = 0;
         uint32_t chb = 0;
         unsigned long long offer = 0;
+        bool skipped = false;
         if (got) {
-            ++st_tasks;
             if (item & CHUNK_FLAG) {
-                ++st_chunks;
                 const int2 c = p.chunk_tab[item & ~CHUNK_FLAG];
                 v = c.x;
                 const long long re = ld_nc_i64(p.row_ptr + v + 1);
@@ -409,6 +495,19 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
             // current cost of the node (Listing 2 line 21), read fresh
             const unsigned L = (unsigned)(tq_ld_relaxed(p.W + v) >> 32);
             offer = ((unsigned long long)(L + 1) << 32) | (unsigned)v;
+            if (!(item & CHUNK_FLAG)) {
+                // expanded-level marker (R7): a vertex already
+                // expanded at a level <= L has offered <= L+1 to every
+                // neighbour, so this token has nothing left to do
+                const int xprev = ld_relaxed_i32(p.xl + v);
+                if (xprev <= (int)L) {
+                    skipped = true;
+                    hi = lo;
+                    nch = 0;
+                } else {
+                    st_relaxed_i32(p.xl + v, (int)L);
+                }
+            }
         }
 
         // ---- DoWorkUnit(): warp-cooperative expansion ----
@@ -416,13 +515,23 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
         const int incl = warp_incl_scan(deg, lane);
         const int total = __shfl_sync(TQ_FULL_MASK, incl, 31);
         const long long ebase = lo - (incl - deg);
+        {
+            const unsigned chm = __ballot_sync(TQ_FULL_MASK, got && (item & CHUNK_FLAG));
+            const unsigned skm = __ballot_sync(TQ_FULL_MASK, skipped);
+            if (lane == 0) {
+                S[ST_TASKS] += __popc(gm);
+                S[ST_CHUNK_TASKS] += __popc(chm);
+                S[ST_SKIPPED] += __popc(skm);
+                S[ST_EDGES] += (unsigned)total;
+            }
+        }
         unsigned cnt = 0;
-        for (int b = 0; b < total; b += 32 * kU) {
-            int32_t u[kU];
-            unsigned long long off[kU];
-            bool val[kU];
+        for (int b = 0; b < total; b += 32 * KU) {
+            int32_t u[KU];
+            unsigned long long off[KU];
+            bool val[KU];
 #pragma unroll
-            for (int j = 0; j < kU; ++j) {
+            for (int j = 0; j < KU; ++j) {
                 const int g = b + j * 32 + (int)lane;
                 val[j] = g < total;
                 const int gg = val[j] ? g : total - 1;
@@ -431,34 +540,62 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
                 off[j] = tq_shfl64(offer, o);
                 u[j] = val[j] ? ld_nc_i32(p.col + eb + gg) : 0;
             }
-            unsigned long long w[kU];
+            // prefilter 1: the byte level mirror (L2-resident; stale values
+            // are never below the true level, R8)
+            unsigned m8[KU];
 #pragma unroll
-            for (int j = 0; j < kU; ++j) w[j] = val[j] ? ld_cg_u64(p.W + u[j]) : 0ull;
-            bool nt[kU];
+            for (int j = 0; j < KU; ++j) m8[j] = val[j] ? ld_cg_u8(p.lvl8 + u[j]) : 0u;
+            bool cand[KU], tie[KU];
 #pragma unroll
-            for (int j = 0; j < kU; ++j) {
+            for (int j = 0; j < KU; ++j) {
+                const unsigned L1 = (unsigned)(off[j] >> 32);
+                const bool known = m8[j] < kLvlSat;  // exact-or-stale-high level
+                tie[j] = val[j] && min_id && known && m8[j] == L1;
+                cand[j] = val[j] && !(known && m8[j] <= L1);
+            }
+            // prefilter 2 (min-id parents only): the packed word, only for
+            // offers that tie on level and may still win on parent id
+            bool any_tie = false;
+#pragma unroll
+            for (int j = 0; j < KU; ++j) any_tie |= tie[j];
+            if (min_id && __any_sync(TQ_FULL_MASK, any_tie)) {
+                unsigned long long w[KU];
+#pragma unroll
+                for (int j = 0; j < KU; ++j) w[j] = tie[j] ? ld_cg_u64(p.W + u[j]) : 0ull;
+#pragma unroll
+                for (int j = 0; j < KU; ++j) cand[j] = cand[j] || (tie[j] && off[j] < w[j]);
+            }
+            bool nt[KU];
+            unsigned n_min = 0, n_reenq = 0;
+#pragma unroll
+            for (int j = 0; j < KU; ++j) {
                 nt[j] = false;
-                if (val[j]) {
-                    ++st_edges;
-                    if (off[j] < w[j]) {  // stale-tolerant prefilter (R4)
-                        const unsigned long long old = atomicMin(p.W + u[j], off[j]);
-                        ++st_min;
-                        if ((old >> 32) > (off[j] >> 32)) {  // level strictly lowered
-                            nt[j] = true;
-                            if ((old >> 32) != 0xffffffffull) ++st_reenq;
-                        }
+                bool re = false;
+                if (cand[j]) {
+                    const unsigned long long old = atomicMin(p.W + u[j], off[j]);
+                    const unsigned L1 = (unsigned)(off[j] >> 32);
+                    if ((old >> 32) > L1) {  // level strictly lowered: (re)discovered
+                        nt[j] = true;
+                        st_u8(p.lvl8 + u[j], L1 < kLvlSat ? L1 : kLvlSat);
+                        re = (old >> 32) != 0xffffffffull;
                     }
                 }
+                n_min += __popc(__ballot_sync(TQ_FULL_MASK, cand[j]));
+                n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, re));
+            }
+            if (lane == 0) {
+                S[ST_MIN_ATOMICS] += n_min;
+                S[ST_REENQUEUES] += n_reenq;
             }
 #pragma unroll
-            for (int j = 0; j < kU; ++j) {
+            for (int j = 0; j < KU; ++j) {
                 const unsigned m = __ballot_sync(TQ_FULL_MASK, nt[j]);
                 if (nt[j]) stage[cnt + __popc(m & tq_lanemask_lt())] = (uint32_t)u[j];
                 cnt += __popc(m);
             }
-            if (cnt > kStageCap - 32 * kU) {
+            if (cnt > kStageCap - 32 * KU) {
                 __syncwarp();
-                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
+                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.exp_flags);
                 __syncwarp();
                 cnt = 0;
             }
@@ -466,7 +603,7 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
 
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
-        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
+        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.exp_flags);
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
         while (hubm) {
@@ -478,35 +615,38 @@ __global__ void __launch_bounds__(kBlock) bfs_persistent_kernel(const BfsParams 
         }
 
         // ---- completion accounting for WorkRemains() (R6) ----
-        bool fin = false;
+        // Done += tasks finished, with release semantics and no round trip:
+        // it is ordered after this warp's Rear reservations; idle warps
+        // compare Done with Rear.
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
-            // lane 0 issued every Rear reservation of this warp, so its
-            // acq_rel add on Done is ordered after them
+            // lane 0 issued every Rear reservation of this warp
             if (lane == 0) {
-                const unsigned nf = __popc(gm);
-                const unsigned long long old = tq_atom_add_acqrel(q.done, nf);
+                if (p.exp_flags & 4)
+                    atomicAdd(q.done, (unsigned long long)__popc(gm));
+                else
+                    tq_red_add_release(q.done, (unsigned long long)__popc(gm));
                 ++st_qatom;
-                fin = old + nf == tq_ld_relaxed(q.rear);
             }
         } else {
             __syncwarp();
             tq_fence_gpu();
             if (got) {
-                const unsigned long long old = tq_atom_add_acqrel(q.done, 1ull);
+                tq_red_add_release(q.done, 1ull);
                 ++st_qatom;
-                fin = old + 1 == tq_ld_relaxed(q.rear);
             }
         }
-        if (__any_sync(TQ_FULL_MASK, fin)) tq_warp_status_set(q, TQ_FINISHED);
     }
 
     // ---- statistics (one atomic per counter per warp) ----
-    const unsigned long long s[8] = {st_tasks, st_chunks, st_edges, st_min,
-                                     st_reenq, st_qatom,  st_fail,  st_empty};
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-        const unsigned long long x = warp_sum(s[k]);
-        if (lane == 0 && x) atomicAdd(p.stats + k, x);
+    {
+        const unsigned long long qa = warp_sum((unsigned long long)st_qatom);
+        const unsigned long long cf = warp_sum((unsigned long long)st_fail);
+        if (lane == 0) {
+            S[ST_QUEUE_ATOMICS] += qa;
+            S[ST_CAS_FAILURES] += cf;
+        }
+        __syncwarp();
+        if (lane < ST_REACHED && S[lane]) atomicAdd(p.stats + lane, S[lane]);
     }
 }
 
@@ -518,8 +658,11 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
 {
     const int64_t n = p.n_vertices;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
         p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
+        p.lvl8[i] = (i == root) ? 0 : 255;
+        p.xl[i] = 0x7fffffff;
+    }
     if (blockIdx.x == 0) {
         if (threadIdx.x < TQ_STATUS_COPIES) p.q.status[threadIdx.x * TQ_STATUS_STRIDE] = TQ_RUNNING;
         if (threadIdx.x < kStatCount) p.stats[threadIdx.x] = 0;
@@ -656,17 +799,29 @@ cudaError_t launch_queue_reset(const tq_device_view &q, cudaStream_t s)
     return cudaGetLastError();
 }
 
-template <int V>
+template <int V, int KU = kU, int MINB = kMinBlocks>
 static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStream_t s)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
-    bfs_persistent_kernel<V><<<blocks, kBlock, 0, s>>>(p);
+    bfs_persistent_kernel<V, KU, MINB><<<blocks, kBlock, 0, s>>>(p);
     return cudaGetLastError();
 }
+
+// experiment instances (TQ_EXP_FLAGS >> 8): unroll depth x min blocks per SM
+#define TQ_EXP_INSTANCES(X) X(1, 8, 1) X(2, 4, 6) X(3, 4, 8) X(4, 8, 6) X(5, 2, 8)
 
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
                                   cudaStream_t s)
 {
+    if (variant == TQ_VARIANT_RF_AN && (p.exp_flags >> 8)) {
+        switch (p.exp_flags >> 8) {
+#define X(id, ku, mb) \
+    case id: return launch_v<TQ_VARIANT_RF_AN, ku, mb>(p, blocks, block, s);
+            TQ_EXP_INSTANCES(X)
+#undef X
+        default: return cudaErrorInvalidValue;
+        }
+    }
     switch (variant) {
     case TQ_VARIANT_RF_AN: return launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
     case TQ_VARIANT_PER_THREAD_AFA: return launch_v<TQ_VARIANT_PER_THREAD_AFA>(p, blocks, block, s);
@@ -679,6 +834,19 @@ cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, i
 cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
+    const char *ef = getenv("TQ_EXP_FLAGS");
+    const unsigned exp = ef ? (unsigned)atoi(ef) >> 8 : 0u;
+    if (variant == TQ_VARIANT_RF_AN && exp) {
+        switch (exp) {
+#define X(id, ku, mb)                                              \
+    case id:                                                       \
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(      \
+            blocks_per_sm, bfs_persistent_kernel<TQ_VARIANT_RF_AN, ku, mb>, kBlock, 0);
+            TQ_EXP_INSTANCES(X)
+#undef X
+        default: return cudaErrorInvalidValue;
+        }
+    }
     switch (variant) {
     case TQ_VARIANT_RF_AN:
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(

@@ -26,6 +26,7 @@ enum StatIndex {
     ST_QUEUE_ATOMICS,
     ST_CAS_FAILURES,
     ST_EMPTY_POLLS,
+    ST_SKIPPED,
     // filled by the unpack kernel
     ST_REACHED,
     ST_DEG_SUM,
@@ -40,10 +41,14 @@ struct BfsParams {
     unsigned long long *W;     // packed (level << 32) | parent, ~0 = unreached
     const int2 *chunk_tab;     // chunk id -> {vertex, k}
     const int32_t *hub_base;   // vertex -> first chunk id (read for hubs only)
+    uint8_t *lvl8;             // byte level mirror (prefilter), 255 = unreached
+    int32_t *xl;               // level at which the vertex was last expanded
     unsigned long long *stats; // kStatCount counters
     int64_t n_vertices;
     int chunk;                 // max edges per token (power of 2)
     int backoff_ns;            // max idle back-off, 0 = none
+    int parent_rule;           // TQ_PARENT_ANY / TQ_PARENT_MIN_ID (include/tq.h)
+    unsigned exp_flags;        // experiments only (TQ_EXP_FLAGS env), 0 in production
     unsigned long long timeout_ns;
 };
 
