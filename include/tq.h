@@ -136,7 +136,7 @@ typedef struct {
     int chunk;          /* sub-task size: max edges per task token (P:153
                            "a fixed number of uniformly complex sub-tasks";
                            P:159 fn3).  Vertices with more edges are split
-                           into chunk tokens.  0 = 256; power of 2 in
+                           into chunk tokens.  0 = 512; power of 2 in
                            [32, 2^16]                                        */
     int variant;        /* tq_variant (RF_AN, PER_THREAD_AFA, CAS_RETRY, AN) */
     void *stream;       /* cudaStream_t                                      */
@@ -150,6 +150,10 @@ typedef struct {
                            TQ_PARENT_MIN_ID (1): the smallest-id neighbour one
                            level up (unique, bit-exact; ~20% slower: level
                            ties must consult the packed word)               */
+    int hub_queue;      /* RF_AN: chunk tokens of high-degree vertices go to a
+                           second RF/AN queue that lane 0 of every warp polls
+                           first (0 = default on, < 0 = off: chunks share the
+                           main queue).  Ignored by the other variants.     */
 } bfs_opts;
 
 enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };

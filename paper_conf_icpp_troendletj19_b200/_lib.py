@@ -38,7 +38,7 @@ class bfs_opts(ctypes.Structure):
     _fields_ = [("capacity", c_u64), ("threads", ctypes.c_int), ("block", ctypes.c_int),
                 ("chunk", ctypes.c_int), ("variant", ctypes.c_int), ("stream", c_vp),
                 ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int),
-                ("parent_rule", ctypes.c_int)]
+                ("parent_rule", ctypes.c_int), ("hub_queue", ctypes.c_int)]
 
 
 class bfs_stats(ctypes.Structure):

@@ -74,10 +74,11 @@ def _csr(row_ptr, col) -> _lib.tq_csr:
 
 
 def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None, timeout_s=0.0,
-          backoff_ns=0, device=0, parents="any") -> _lib.bfs_opts:
+          backoff_ns=0, device=0, parents="any", hub_queue=True) -> _lib.bfs_opts:
     return _lib.bfs_opts(int(capacity), int(threads), int(block), int(chunk), _variant(variant),
                          stream, float(timeout_s), int(backoff_ns), int(device),
-                         _lib.PARENT_RULES[parents] if isinstance(parents, str) else int(parents))
+                         _lib.PARENT_RULES[parents] if isinstance(parents, str) else int(parents),
+                         0 if hub_queue else -1)
 
 
 def _stats_dict(st: _lib.bfs_stats) -> dict:
@@ -93,7 +94,8 @@ def _empty_like_graph(row_ptr, n):
 
 def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool = True,
         variant="rf_an", capacity: int = 0, threads: int = 0, chunk: int = 0, stream=None,
-        timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0, parents="any"):
+        timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0, parents="any",
+        hub_queue: bool = True):
     """One-shot `bfs_run_ex`: returns (level, parent, stats).
 
     Graph arrays may be CUDA tensors (used in place) or host numpy arrays
@@ -108,7 +110,7 @@ def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool =
         parent = _empty_like_graph(row_ptr, n)
     o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
               backoff_ns, row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device,
-              parents)
+              parents, hub_queue)
     st = _lib.bfs_stats()
     check(lib().bfs_run_ex(ctypes.byref(g), int(root), _ptr(level), _ptr(parent), ctypes.byref(o),
                            ctypes.byref(st)), "bfs_run_ex")
@@ -124,14 +126,14 @@ class BfsPlan:
 
     def __init__(self, row_ptr, col, *, variant="rf_an", capacity: int = 0, threads: int = 0,
                  chunk: int = 0, stream=None, timeout_s: float = 0.0, backoff_ns: int = 0,
-                 device: int = 0, parents="any"):
+                 device: int = 0, parents="any", hub_queue: bool = True):
         self._keep = (row_ptr, col)  # device arrays must outlive the plan
         self._g = _csr(row_ptr, col)
         self.n_vertices = self._g.n_vertices
         self.nnz = self._g.nnz
         self.device = row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device
         o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
-                  backoff_ns, self.device, parents)
+                  backoff_ns, self.device, parents, hub_queue)
         h = ctypes.c_void_p()
         check(lib().bfs_plan_create(ctypes.byref(self._g), ctypes.byref(o), ctypes.byref(h)),
               "bfs_plan_create")

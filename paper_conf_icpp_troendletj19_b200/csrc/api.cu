@@ -110,6 +110,9 @@ struct bfs_plan {
     int2 *chunk_tab = nullptr;
     int64_t n_chunks = 0;
     tq_queue *q = nullptr;
+    tq_queue *q1 = nullptr;                   // chunk queue (RF/AN hub sub-tasks)
+    bool hub_queue = false;
+    unsigned long long next_ticket1 = 0;
     unsigned long long *stats = nullptr;      // device, kStatCount
     unsigned long long *stats_h = nullptr;    // pinned
     unsigned long long next_ticket = 0;
@@ -255,6 +258,7 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     cudaFree(p->out_scratch);
     if (p->stats_h) cudaFreeHost(p->stats_h);
     tq_destroy(p->q);
+    tq_destroy(p->q1);
     delete p;
     return TQ_OK;
 }
@@ -270,7 +274,7 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (n < 1 || n >= (1ll << 31) || nnz < 0 || !gph->row_ptr || (nnz > 0 && !gph->col))
         return TQ_ERR_INVALID;
     if (o.variant < TQ_VARIANT_RF_AN || o.variant > TQ_VARIANT_AN) return TQ_ERR_UNSUPPORTED;
-    int chunk = o.chunk ? o.chunk : 256;
+    int chunk = o.chunk ? o.chunk : 512;
     if (chunk < 32 || chunk > 65536 || (chunk & (chunk - 1))) return TQ_ERR_INVALID;
     const int block = o.block ? o.block : 256;
     if (block != 256) return TQ_ERR_UNSUPPORTED;
@@ -335,6 +339,16 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (!o.capacity && cap < (1ull << 16)) cap = 1ull << 16;
     tq_status st = tq_create(cap, gdev, &p->q);
     if (st != TQ_OK) return fail(st);
+    // chunk queue (RF/AN only): holds at most the chunks of the hubs being
+    // expanded; 2x the chunk count covers a re-expansion of every hub
+    p->hub_queue = p->variant == TQ_VARIANT_RF_AN && o.hub_queue >= 0 && p->n_chunks > 0;
+    if (p->hub_queue) {
+        uint64_t cap1 = next_pow2((uint64_t)(2 * p->n_chunks));
+        if (cap1 < (1ull << 16)) cap1 = 1ull << 16;
+        if (o.capacity && cap1 > next_pow2(o.capacity)) cap1 = next_pow2(o.capacity);
+        st = tq_create(cap1, gdev, &p->q1);
+        if (st != TQ_OK) return fail(st);
+    }
 
     int per_sm = 0;
     e = bfs_occupancy(p->variant, block, &per_sm);
@@ -358,12 +372,22 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     cudaStream_t s = p->stream;
     if (p->dirty) {
         tq_status st = tq_reset(p->q, s);
+        if (st == TQ_OK && p->q1) st = tq_reset(p->q1, s);
         if (st != TQ_OK) return st;
         p->next_ticket = 0;
+        p->next_ticket1 = 0;
         p->dirty = false;
     }
     BfsParams bp{};
     bp.q = p->q->view;
+    if (p->hub_queue) {
+        bp.q1 = p->q1->view;
+        bp.q1.status = p->q->view.status;  // one status word for both queues
+        bp.hub_queue = 1;
+        // chunk-queue ticket holders per warp: lanes 0 and 16 (measured on
+        // B200 kron24 over 1/2/4/8 holders x chunk 256..1024: 2 x 512 best)
+        bp.q1_lanes = 0x00010001u;
+    }
     bp.row_ptr = p->row_ptr;
     bp.col = p->col;
     bp.W = p->W;
@@ -380,7 +404,7 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
 
     CK(cudaEventRecord(p->ev[0], s));
-    CK(launch_bfs_init(bp, root, p->next_ticket, s));
+    CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));
     CK(cudaEventRecord(p->ev[1], s));
     CK(launch_bfs_persistent(p->variant, bp, p->blocks, p->block, s));
     CK(cudaEventRecord(p->ev[2], s));
@@ -388,20 +412,22 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     CK(cudaEventRecord(p->ev[3], s));
     CK(cudaMemcpyAsync(p->stats_h, p->stats, kStatCount * sizeof(unsigned long long),
                        cudaMemcpyDeviceToHost, s));
-    unsigned long long ctr[3] = {0, 0, 0};
+    unsigned long long ctr[4] = {0, 0, 0, 0};
     unsigned status = 0;
     CK(cudaMemcpyAsync(&ctr[0], p->q->view.front, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&ctr[1], p->q->view.rear, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&ctr[2], p->q->view.done, 8, cudaMemcpyDeviceToHost, s));
+    if (p->hub_queue) CK(cudaMemcpyAsync(&ctr[3], p->q1->view.rear, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&status, p->q->view.status, 4, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
 
-    const unsigned long long t0 = p->next_ticket;
+    const unsigned long long t0 = p->next_ticket, t1 = p->next_ticket1;
     if (status == TQ_FINISHED) {
         // every reserved ticket below Rear was taken; slots of tickets
         // [Rear, Rear + C) all hold "empty for t", so the next run can start
-        // at Rear without an O(C) reset
+        // at Rear without an O(C) reset (both queues)
         p->next_ticket = ctr[1];
+        if (p->hub_queue) p->next_ticket1 = ctr[3];
     } else {
         p->dirty = true;
     }
@@ -424,7 +450,7 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
         stats->reached = h[ST_REACHED];
         stats->traversed_edges = h[ST_DEG_SUM] / 2;
         stats->max_level = (int32_t)h[ST_MAX_LEVEL];
-        stats->tickets = ctr[1] - t0;
+        stats->tickets = (ctr[1] - t0) + (p->hub_queue ? ctr[3] - t1 : 0ull);
         stats->skipped_tasks = h[ST_SKIPPED];
         stats->persistent_threads = p->blocks * p->block;
     }

@@ -377,17 +377,33 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     // atomic's latency hides behind the expansion.
     unsigned pend_base = 0;  // lane 0: (low half of the) base of the in-flight reservation
     unsigned pend_mask = 0;  // warp-uniform: lanes waiting for it
+    // Chunk queue: a second RF/AN queue holding
+    // only chunk tokens; lane 0 of every warp holds one ticket in it and
+    // polls it before its main-queue ticket, so a hub's chunks are expanded
+    // by consecutive warps right after the hub is dequeued.
+    const bool hubq = VARIANT == TQ_VARIANT_RF_AN && p.hub_queue;
+    const tq_device_view q1 = p.q1;
+    // lanes holding a chunk-queue ticket (warp-uniform mask, e.g. lanes 0,8,16,24)
+    const unsigned q1_lanes = hubq ? p.q1_lanes : 0u;
+    const bool q1_lane = (q1_lanes >> lane) & 1u;
+    unsigned tk1 = 0, pend1_base = 0, pend1_mask = 0;
+    bool have1 = false;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
         pend_mask = TQ_FULL_MASK;
+        pend1_mask = q1_lanes;
         if (lane == 0) {
             pend_base = (unsigned)tq_atom_add(q.front, 32ull);
             ++st_qatom;
+            if (hubq) {
+                pend1_base = (unsigned)tq_atom_add(q1.front, (unsigned long long)__popc(q1_lanes));
+                ++st_qatom;
+            }
         }
     }
 
     for (;;) {
         // ---- Listing 1 + Listing 2: GetWorkToken() ----
-        bool got = false;
+        bool got = false, got1 = false;
         uint32_t item = 0;
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
             if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
@@ -399,12 +415,27 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     }
                     pend_mask = 0;
                 }
+                if (pend1_mask) {
+                    const unsigned base = __shfl_sync(TQ_FULL_MASK, pend1_base, 0);
+                    if (pend1_mask >> lane & 1u) {
+                        tk1 = base + __popc(pend1_mask & tq_lanemask_lt());
+                        have1 = true;
+                    }
+                    pend1_mask = 0;
+                }
+                if (q1_lane) {
+                    if (have1) {
+                        const unsigned long long sv = tq_ld_relaxed(q1.slots + (tk1 & q1.mask));
+                        got1 = (unsigned)sv == tk1 + 1u;
+                        item = (uint32_t)(sv >> 32);
+                    }
+                }
             } else if (!have) {
                 tk = (unsigned)tq_atom_add(q.front, 1ull);
                 have = true;
                 ++st_qatom;
             }
-            if (have) {  // Listing 2 lines 3-5: non-atomic arrival check
+            if (have && !got1) {  // Listing 2 lines 3-5: non-atomic arrival check
                 const unsigned long long sv = tq_ld_relaxed(q.slots + (tk & q.mask));
                 got = (unsigned)sv == tk + 1u;
                 item = (uint32_t)(sv >> 32);
@@ -422,6 +453,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 got = true;
             }
         }
+        const bool got0 = got;  // token from the main queue
+        got = got || got1;
         const unsigned gm = __ballot_sync(TQ_FULL_MASK, got);
         if (gm == 0) {
             // ---- idle work cycle: Algorithm 1 line 1, WorkRemains() ----
@@ -434,7 +467,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     // Done is read before Rear (R6): done(t1) ==
                     // rear(t2), t1 < t2, implies nothing is queued or in flight
                     const unsigned long long d = tq_ld_acquire(q.done);
-                    fin = d == tq_ld_relaxed(q.rear);
+                    fin = d == tq_ld_relaxed(q.rear) + (hubq ? tq_ld_relaxed(q1.rear) : 0ull);
                     if (!fin && tq_globaltimer() > wdeadline[threadIdx.x >> 5])
                         tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
                 }
@@ -454,17 +487,28 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         if (((++busy) & 63) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
         if (!(p.exp_flags & 1)) tq_fence_gpu();  // acquire: the producer's W update is visible now
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
-            if (got) {  // put the slot back to dna for the next lap
+            if (got0) {  // put the slot back to dna for the next lap
                 tq_st_relaxed(q.slots + (tk & q.mask), (unsigned long long)(tk + cap32));
                 have = false;
             }
         }
         if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
             // first half of the next dequeue (Listing 1 lines 12-14)
-            pend_mask = gm;
+            pend_mask = __ballot_sync(TQ_FULL_MASK, got0);
+            pend1_mask = __ballot_sync(TQ_FULL_MASK, got1);
+            if (got1) {
+                tq_st_relaxed(q1.slots + (tk1 & q1.mask), (unsigned long long)(tk1 + (unsigned)(q1.mask + 1)));
+                have1 = false;
+            }
             if (lane == 0) {
-                pend_base = (unsigned)tq_atom_add(q.front, (unsigned long long)__popc(gm));
-                ++st_qatom;
+                if (pend_mask) {
+                    pend_base = (unsigned)tq_atom_add(q.front, (unsigned long long)__popc(pend_mask));
+                    ++st_qatom;
+                }
+                if (pend1_mask) {
+                    pend1_base = (unsigned)tq_atom_add(q1.front, (unsigned long long)__popc(pend1_mask));
+                    ++st_qatom;
+                }
             }
         }
 
@@ -611,7 +655,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             hubm &= hubm - 1;
             const unsigned n = __shfl_sync(TQ_FULL_MASK, nch, h);
             const uint32_t first = __shfl_sync(TQ_FULL_MASK, chb, h);
-            enqueue_chunks<VARIANT>(q, first, n, lane, &st_qatom, &st_fail);
+            enqueue_chunks<VARIANT>(hubq ? q1 : q, first, n, lane, &st_qatom, &st_fail);
         }
 
         // ---- completion accounting for WorkRemains() (R6) ----
@@ -654,7 +698,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 // a2: state + queue init for one run.  W[:] = unreached, W[root] = (0, root);
 // the root is published at ticket t0 (Front = Done = t0, Rear = t0 + 1).
 // ---------------------------------------------------------------------------
-__global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long long t0)
+__global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long long t0,
+                                unsigned long long t1)
 {
     const int64_t n = p.n_vertices;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -671,7 +716,13 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
                 ((unsigned long long)(uint32_t)root << 32) | (unsigned)(t0 + 1);
             *p.q.front = t0;
             *p.q.rear = t0 + 1;
-            *p.q.done = t0;
+            // Done counts tasks of both queues: termination is
+            // done == rear(main) + rear(chunk queue)
+            *p.q.done = t0 + (p.hub_queue ? t1 : 0ull);
+            if (p.hub_queue) {
+                *p.q1.front = t1;
+                *p.q1.rear = t1;
+            }
         }
     }
 }
@@ -781,9 +832,10 @@ static int grid_for(int64_t n, int block)
     return (int)(want < 1 ? 1 : (want < cap ? want : cap));
 }
 
-cudaError_t launch_bfs_init(const BfsParams &p, int32_t root, unsigned long long t0, cudaStream_t s)
+cudaError_t launch_bfs_init(const BfsParams &p, int32_t root, unsigned long long t0,
+                            unsigned long long t1, cudaStream_t s)
 {
-    bfs_init_kernel<<<grid_for(p.n_vertices, 256), 256, 0, s>>>(p, root, t0);
+    bfs_init_kernel<<<grid_for(p.n_vertices, 256), 256, 0, s>>>(p, root, t0, t1);
     return cudaGetLastError();
 }
 

@@ -35,7 +35,10 @@ enum StatIndex {
 };
 
 struct BfsParams {
-    tq_device_view q;
+    tq_device_view q;          // main queue: vertex tokens (and chunk tokens if !hub_queue)
+    tq_device_view q1;         // chunk queue (hub sub-tasks), valid if hub_queue
+    int hub_queue;             // RF/AN only: chunk tokens go to q1, polled first
+    unsigned q1_lanes;         // lanes of each warp that hold a q1 ticket
     const int64_t *row_ptr;
     const int32_t *col;
     unsigned long long *W;     // packed (level << 32) | parent, ~0 = unreached
@@ -53,7 +56,8 @@ struct BfsParams {
 };
 
 // bfs.cu
-cudaError_t launch_bfs_init(const BfsParams &p, int32_t root, unsigned long long t0, cudaStream_t s);
+cudaError_t launch_bfs_init(const BfsParams &p, int32_t root, unsigned long long t0,
+                            unsigned long long t1, cudaStream_t s);
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
                                   cudaStream_t s);
 cudaError_t launch_bfs_unpack(const BfsParams &p, int32_t *level, int32_t *parent, cudaStream_t s);

@@ -18,7 +18,8 @@ ap.add_argument("--threads", default="0")
 ap.add_argument("--backoff", default="0")
 ap.add_argument("--variants", default="rf_an")
 ap.add_argument("--roots", type=int, default=2)
-ap.add_argument("--parents", default="min_id")
+ap.add_argument("--parents", default="any")
+ap.add_argument("--hubq", default="1")
 args = ap.parse_args()
 kind, a, ef, nr = bench.WORKLOADS[args.workload]
 dev = torch.device("cuda", 0)
@@ -30,7 +31,7 @@ pa = torch.empty(n, dtype=torch.int32, device=dev)
 for var, ch, th, bo in itertools.product(args.variants.split(","), map(int, args.chunks.split(",")),
                                          map(int, args.threads.split(",")), map(int, args.backoff.split(","))):
     plan = tq.BfsPlan(rp, col, variant=var, chunk=ch, threads=th, backoff_ns=bo, timeout_s=60,
-                      parents=args.parents)
+                      parents=args.parents, hub_queue=args.hubq == "1")
     plan.run(roots[0], lv, pa)
     for r in roots:
         st = plan.run(r, lv, pa)
