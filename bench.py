@@ -148,6 +148,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=20.0)
+    ap.add_argument("--parents", default="any", choices=["any", "min_id"])
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", 0))
@@ -173,65 +174,50 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     import paper_conf_icpp_troendletj19_b200 as tq
+    from paper_conf_icpp_troendletj19_b200 import multiroot
 
     # ---- inputs (not timed): generated on the device, replicated per rank ----
     t_gen = time.time()
     row_ptr, col = make_graph(kind, a, ef, dev)
     rp_host = row_ptr.cpu().numpy()
     roots = pick_roots(kind, rp_host, n_roots)
-    mine = roots[rank * len(roots) // world:(rank + 1) * len(roots) // world]
+    mine = multiroot.split_roots(roots, rank, world)
     n = int(row_ptr.numel()) - 1
     t_gen = time.time() - t_gen
 
     stream = torch.cuda.current_stream(dev)
-    plan = tq.BfsPlan(row_ptr, col, variant=args.variant, stream=stream, device=local)
+    plan = tq.BfsPlan(row_ptr, col, variant=args.variant, stream=stream, device=local,
+                      parents=args.parents)
     level = torch.empty(n, dtype=torch.int32, device=dev)
     parent = torch.empty(n, dtype=torch.int32, device=dev)
 
-    def step():
-        sts = []
-        for r in mine:
-            sts.append(plan.run(r, level, parent))
-        return sts
+    def run_root(r):
+        return plan.run(r, level, parent)
 
-    for _ in range(args.warmup):
-        step()
+    multiroot.run_local(run_root, mine, steps=args.warmup)
 
     # ---- timed region: K steps, barrier + sync on both sides, device events ----
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    all_stats = []
     with ClockSampler(local) as clk:
         e0.record(stream)
-        for _ in range(args.steps):
-            all_stats.extend(step())
+        all_stats = multiroot.run_local(run_root, mine, steps=args.steps)
         e1.record(stream)
         torch.cuda.synchronize(dev)
     if dist:
         dist.barrier()
     ms_total = e0.elapsed_time(e1)
-    te_local = sum(s["traversed_edges"] for s in all_stats)
-    reached_local = sum(s["reached"] for s in all_stats)
-    kern_ms_local = sum(s["ms_kernel"] for s in all_stats)
-    launches_local = 3 * len(all_stats)
 
-    # NCCL gather of per-rank stats (the only collective; outside the data path)
-    vec = torch.tensor([ms_total, te_local, reached_local, kern_ms_local, launches_local,
-                        len(all_stats)], dtype=torch.float64, device=dev)
-    if dist:
-        out = torch.empty(world * vec.numel(), dtype=torch.float64, device=dev)
-        dist.all_gather_into_tensor(out, vec)
-        allv = out.view(world, -1).cpu().numpy()
-    else:
-        allv = vec.view(1, -1).cpu().numpy()
-    ms_max = float(allv[:, 0].max())
-    te_all = float(allv[:, 1].sum())
-    reached_all = float(allv[:, 2].sum())
-    kern_ms_all = float(allv[:, 3].sum())
-    launches = int(allv[:, 4].sum())
-    runs_all = int(allv[:, 5].sum())
+    # NCCL all-gather of per-rank stats (the only collective; outside the data path)
+    agg = multiroot.aggregate(multiroot.gather(multiroot.local_vector(all_stats, ms_total), dist, dev))
+    ms_max = agg["ms"]
+    te_all = agg["traversed_edges"]
+    reached_all = agg["reached"]
+    kern_ms_all = agg["ms_kernel_sum"]
+    launches = int(agg["launches"])
+    runs_all = int(agg["runs"])
 
     gteps = te_all / (ms_max * 1e-3) / 1e9
     ms_per_step = ms_max / args.steps
@@ -263,7 +249,8 @@ def main():
         t0 = time.perf_counter()
         te_e2e = 0
         for _ in range(args.steps):
-            with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=stream, device=local) as hp:
+            with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=stream, device=local,
+                            parents=args.parents) as hp:
                 for r in mine:
                     s = hp.run(r, lv_np, pa_np)
                     te_e2e += s["traversed_edges"]
@@ -288,7 +275,7 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu:
         col_host = col.cpu().numpy()
         teps, done, sec, lv0 = cpu_oracle_sample(rp_host, col_host, mine, args.cpu_budget)
-        plan2 = tq.BfsPlan(row_ptr, col, variant=args.variant, device=local)
+        plan2 = tq.BfsPlan(row_ptr, col, variant=args.variant, device=local, parents=args.parents)
         plan2.run(done[0], level, parent)
         parity = bool(np.array_equal(level.cpu().numpy(), lv0))
         plan2.close()

@@ -1,0 +1,81 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py
+times (default options: RF/AN, chunk queue, parents='any', full occupancy).
+
+* config 3, grid 4096 x 4096 from the corner: levels against the closed form
+  level(r, c) = r + c (every vertex), parents valid; with the min-id rule the
+  parents against the closed form v - 4096 (r > 0) / v - 1.
+* config 4, Kronecker scale 24: every level against the oracle for 2 roots.
+* config 5, Kronecker scale 26: every level against the oracle for 1 root.
+"""
+import numpy as np
+import pytest
+
+import oracle
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+@pytest.fixture(scope="module")
+def tq():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_icpp_troendletj19_b200 as m
+    return m
+
+
+def test_grid4096_closed_form(tq):
+    import torch
+    import inputs.gpu as gg
+    rows = 4096
+    rp, col = gg.grid_csr_cuda(rows)
+    n = rows * rows
+    v = torch.arange(n, device="cuda", dtype=torch.int64)
+    r, c = v // rows, v % rows
+    for parents in ("any", "min_id"):
+        level, parent, st = tq.bfs(rp, col, 0, parents=parents)
+        assert torch.equal(level.long(), r + c)
+        lp = level.long()[parent.long()]
+        assert torch.equal(lp[1:], level.long()[1:] - 1) and int(parent[0]) == 0
+        if parents == "min_id":
+            exp = torch.where(r > 0, v - rows, v - 1)
+            exp[0] = 0
+            assert torch.equal(parent.long(), exp)
+        assert st["traversed_edges"] == 2 * rows * (rows - 1) and st["max_level"] == 2 * rows - 2
+
+
+def _kron_check(tq, scale, n_roots):
+    import torch
+    import inputs.gpu as gg
+    from inputs import sample_roots
+    rp, col = gg.kronecker_csr_cuda(scale, 16, 1)
+    rp_h, col_h = rp.cpu().numpy(), col.cpu().numpy()
+    n = rp.numel() - 1
+    level = torch.empty(n, dtype=torch.int32, device="cuda")
+    parent = torch.empty_like(level)
+    with tq.BfsPlan(rp, col) as plan:
+        for root in sample_roots(rp_h, n_roots, 2):
+            st = plan.run(int(root), level, parent)
+            lv_o, _, info = oracle.bfs(rp_h, col_h, int(root), parents=False)
+            lv = level.cpu().numpy()
+            bad = np.flatnonzero(lv != lv_o)
+            assert bad.size == 0, f"{bad.size} level mismatches"
+            pa = parent.cpu().numpy()
+            reached = lv_o > 0
+            assert np.all(lv_o[pa[reached]] == lv_o[reached] - 1)
+            assert st["traversed_edges"] == info["traversed_edges"]
+            assert st["reached"] == info["reached"]
+
+
+def test_kron24_levels_identical(tq):
+    _kron_check(tq, 24, 2)
+
+
+def test_kron26_levels_identical(tq):
+    _kron_check(tq, 26, 1)
+
+
+def test_queue_bench_full_size_conserves(tq):
+    from inputs import fingerprint, item_of
+    for variant in ("rf_an", "per_thread_afa", "cas_retry", "an"):
+        r = tq.queue_bench(variant, warps=0, batch=32, items=1 << 24, capacity=1 << 20, seed=3)
+        assert (r["deq"], r["sum_deq"], r["xor_deq"]) == fingerprint(item_of(3, np.arange(r["items"])))
