@@ -192,7 +192,7 @@ def main():
     parent = torch.empty(n, dtype=torch.int32, device=dev)
 
     def run_root(r):
-        return plan.run(r, level, parent)
+        return plan.run(r, level, parent, grow_on_full=True)
 
     multiroot.run_local(run_root, mine, steps=args.warmup)
 
@@ -209,6 +209,7 @@ def main():
     if dist:
         dist.barrier()
     ms_total = e0.elapsed_time(e1)
+    regrows = plan.regrows
 
     # NCCL all-gather of per-rank stats (the only collective; outside the data path)
     agg = multiroot.aggregate(multiroot.gather(multiroot.local_vector(all_stats, ms_total), dist, dev))
@@ -241,7 +242,7 @@ def main():
         lv_pin = torch.empty(n, dtype=torch.int32, pin_memory=True)
         pa_pin = torch.empty(n, dtype=torch.int32, pin_memory=True)
         rp_np, col_np, lv_np, pa_np = rp_pin.numpy(), col_pin.numpy(), lv_pin.numpy(), pa_pin.numpy()
-        del plan
+        plan.close()
         torch.cuda.empty_cache()
         if dist:
             dist.barrier()
@@ -314,6 +315,7 @@ def main():
             "clocks": clk.summary(),
             "parity_sampled_root_levels_identical": parity,
             "graph_gen_s": round(t_gen, 2),
+            "queue_regrows": regrows,
         }
         print(json.dumps(line), flush=True)
     if dist:

@@ -132,18 +132,34 @@ class BfsPlan:
         self.n_vertices = self._g.n_vertices
         self.nnz = self._g.nnz
         self.device = row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device
-        o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
-                  backoff_ns, self.device, parents, hub_queue)
+        self._opts = o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr),
+                               timeout_s, backoff_ns, self.device, parents, hub_queue)
+        self.regrows = 0
+        self._h = None
+        self._create()
+
+    def _create(self):
         h = ctypes.c_void_p()
-        check(lib().bfs_plan_create(ctypes.byref(self._g), ctypes.byref(o), ctypes.byref(h)),
+        check(lib().bfs_plan_create(ctypes.byref(self._g), ctypes.byref(self._opts), ctypes.byref(h)),
               "bfs_plan_create")
         self._h = h
 
-    def run(self, root: int, level=None, parent=None) -> dict:
-        st = _lib.bfs_stats()
-        check(lib().bfs_plan_run(self._h, int(root), _ptr(level), _ptr(parent), ctypes.byref(st)),
-              "bfs_plan_run")
-        return _stats_dict(st)
+    def run(self, root: int, level=None, parent=None, grow_on_full: bool = False) -> dict:
+        """One BFS. With grow_on_full, a queue-full abort (TQ_ERR_QUEUE_FULL)
+        is answered as the paper suggests: re-create the plan with
+        twice the queue capacity and run again (counted in `regrows`)."""
+        while True:
+            st = _lib.bfs_stats()
+            status = lib().bfs_plan_run(self._h, int(root), _ptr(level), _ptr(parent), ctypes.byref(st))
+            if status == _lib.TQ_ERR_QUEUE_FULL and grow_on_full:
+                cap = self._opts.capacity or 2 * max(self.n_vertices, 1 << 15)
+                self._opts.capacity = 2 * max(cap, 1 << 16)
+                self.close()
+                self._create()
+                self.regrows += 1
+                continue
+            check(status, "bfs_plan_run")
+            return _stats_dict(st)
 
     def close(self):
         h = getattr(self, "_h", None)

@@ -106,7 +106,7 @@ struct bfs_plan {
     unsigned long long *W = nullptr;
     int32_t *hub_base = nullptr;
     uint8_t *lvl8 = nullptr;
-    int32_t *xl = nullptr;
+    uint8_t *x8 = nullptr;
     int2 *chunk_tab = nullptr;
     int64_t n_chunks = 0;
     tq_queue *q = nullptr;
@@ -252,7 +252,7 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     cudaFree(p->W);
     cudaFree(p->hub_base);
     cudaFree(p->lvl8);
-    cudaFree(p->xl);
+    cudaFree(p->x8);
     cudaFree(p->chunk_tab);
     cudaFree(p->stats);
     cudaFree(p->out_scratch);
@@ -325,7 +325,7 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     e = cudaMalloc(&p->W, (size_t)n * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMalloc(&p->hub_base, (size_t)n * sizeof(int32_t));
     if (e == cudaSuccess) e = cudaMalloc(&p->lvl8, (size_t)n);
-    if (e == cudaSuccess) e = cudaMalloc(&p->xl, (size_t)n * sizeof(int32_t));
+    if (e == cudaSuccess) e = cudaMalloc(&p->x8, (size_t)n);
     if (e == cudaSuccess) e = cudaMalloc(&p->stats, kStatCount * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
     for (auto &ev : p->ev)
@@ -339,12 +339,13 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (!o.capacity && cap < (1ull << 16)) cap = 1ull << 16;
     tq_status st = tq_create(cap, gdev, &p->q);
     if (st != TQ_OK) return fail(st);
-    // chunk queue (RF/AN only): holds at most the chunks of the hubs being
-    // expanded; 2x the chunk count covers a re-expansion of every hub
+    // chunk queue (RF/AN only): a hub emits its chunks at every expansion
+    // (one per distinct level, R7); 4x the chunk count, at least 2^20 slots
+    // (8 MiB), leaves room for bursts while consumers lag (e.g. under ncu)
     p->hub_queue = p->variant == TQ_VARIANT_RF_AN && o.hub_queue >= 0 && p->n_chunks > 0;
     if (p->hub_queue) {
-        uint64_t cap1 = next_pow2((uint64_t)(2 * p->n_chunks));
-        if (cap1 < (1ull << 16)) cap1 = 1ull << 16;
+        uint64_t cap1 = next_pow2((uint64_t)(4 * p->n_chunks));
+        if (cap1 < (1ull << 20)) cap1 = 1ull << 20;
         if (o.capacity && cap1 > next_pow2(o.capacity)) cap1 = next_pow2(o.capacity);
         st = tq_create(cap1, gdev, &p->q1);
         if (st != TQ_OK) return fail(st);
@@ -394,7 +395,7 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     bp.chunk_tab = p->chunk_tab;
     bp.hub_base = p->hub_base;
     bp.lvl8 = p->lvl8;
-    bp.xl = p->xl;
+    bp.x8 = p->x8;
     bp.parent_rule = p->parent_rule;
     bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;
     bp.stats = p->stats;

@@ -52,10 +52,24 @@ __device__ __forceinline__ unsigned long long ld_cg_u64(const unsigned long long
     asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p));
     return v;
 }
-__device__ __forceinline__ int32_t ld_nc_i32(const int32_t *p)
+// L2 eviction policies (createpolicy, sm_80+): the col stream is read once
+// per expansion and must not evict the L2-resident byte mirror.
+__device__ __forceinline__ unsigned long long l2_policy_evict_first()
+{
+    unsigned long long pol;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ unsigned long long l2_policy_evict_last()
+{
+    unsigned long long pol;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ int32_t ld_nc_i32(const int32_t *p, unsigned long long pol)
 {
     int32_t v;
-    asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
 __device__ __forceinline__ int64_t ld_nc_i64(const int64_t *p)
@@ -65,10 +79,16 @@ __device__ __forceinline__ int64_t ld_nc_i64(const int64_t *p)
     return v;
 }
 
-__device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p)
+__device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long long pol)
 {
     unsigned v;
-    asm volatile("ld.global.cg.u8 %0, [%1];" : "=r"(v) : "l"(p));
+    asm volatile("ld.global.cg.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ unsigned ld_relaxed_u8(const uint8_t *p)
+{
+    unsigned v;
+    asm volatile("ld.relaxed.gpu.global.u8 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ void st_u8(uint8_t *p, unsigned v)
@@ -542,14 +562,16 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             if (!(item & CHUNK_FLAG)) {
                 // expanded-level marker (R7): a vertex already
                 // expanded at a level <= L has offered <= L+1 to every
-                // neighbour, so this token has nothing left to do
-                const int xprev = ld_relaxed_i32(p.xl + v);
-                if (xprev <= (int)L) {
+                // neighbour, so this token has nothing left to do.  A byte,
+                // saturating like the mirror (254 = "expanded at >= 254",
+                // which never skips).
+                const unsigned xprev = ld_relaxed_u8(p.x8 + v);
+                if (xprev < kLvlSat && xprev <= L) {
                     skipped = true;
                     hi = lo;
                     nch = 0;
                 } else {
-                    st_relaxed_i32(p.xl + v, (int)L);
+                    st_u8(p.x8 + v, L < kLvlSat ? L : kLvlSat);
                 }
             }
         }
@@ -570,6 +592,12 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
         }
         unsigned cnt = 0;
+        const unsigned long long pol_stream = l2_policy_evict_first();
+        const unsigned long long pol_keep = l2_policy_evict_last();
+        // Edge -> token map: lane l takes concatenated edges b + 32j + l; its
+        // token is found by a 5-step shuffle binary search over the lanes'
+        // inclusive prefix sums (a shared-memory prefix-max map was measured
+        // and was not faster).
         for (int b = 0; b < total; b += 32 * KU) {
             int32_t u[KU];
             unsigned long long off[KU];
@@ -582,13 +610,13 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 const int o = owner_of(incl, gg);
                 const long long eb = (long long)tq_shfl64((unsigned long long)ebase, o);
                 off[j] = tq_shfl64(offer, o);
-                u[j] = val[j] ? ld_nc_i32(p.col + eb + gg) : 0;
+                u[j] = val[j] ? ld_nc_i32(p.col + eb + gg, pol_stream) : 0;
             }
             // prefilter 1: the byte level mirror (L2-resident; stale values
             // are never below the true level, R8)
             unsigned m8[KU];
 #pragma unroll
-            for (int j = 0; j < KU; ++j) m8[j] = val[j] ? ld_cg_u8(p.lvl8 + u[j]) : 0u;
+            for (int j = 0; j < KU; ++j) m8[j] = val[j] ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : 0u;
             bool cand[KU], tie[KU];
 #pragma unroll
             for (int j = 0; j < KU; ++j) {
@@ -706,7 +734,7 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
         p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
         p.lvl8[i] = (i == root) ? 0 : 255;
-        p.xl[i] = 0x7fffffff;
+        p.x8[i] = 255;
     }
     if (blockIdx.x == 0) {
         if (threadIdx.x < TQ_STATUS_COPIES) p.q.status[threadIdx.x * TQ_STATUS_STRIDE] = TQ_RUNNING;
@@ -859,8 +887,8 @@ static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStrea
     return cudaGetLastError();
 }
 
-// experiment instances (TQ_EXP_FLAGS >> 8): unroll depth x min blocks per SM
-#define TQ_EXP_INSTANCES(X) X(1, 8, 1) X(2, 4, 6) X(3, 4, 8) X(4, 8, 6) X(5, 2, 8)
+// tuning instances (TQ_EXP_FLAGS >> 8): resident blocks per SM
+#define TQ_EXP_INSTANCES(X) X(1, 4, 4) X(2, 4, 5) X(3, 4, 7) X(4, 4, 8)
 
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
                                   cudaStream_t s)

@@ -45,7 +45,7 @@ struct BfsParams {
     const int2 *chunk_tab;     // chunk id -> {vertex, k}
     const int32_t *hub_base;   // vertex -> first chunk id (read for hubs only)
     uint8_t *lvl8;             // byte level mirror (prefilter), 255 = unreached
-    int32_t *xl;               // level at which the vertex was last expanded
+    uint8_t *x8;               // level at which the vertex was expanded (saturating byte)
     unsigned long long *stats; // kStatCount counters
     int64_t n_vertices;
     int chunk;                 // max edges per token (power of 2)

@@ -170,6 +170,19 @@ def test_queue_full_aborts_and_retry_succeeds(tq):
     check_against_oracle(g, root, level, parent, st)
 
 
+def test_grow_on_full_retries_with_larger_queue(tq):
+    g = kronecker_csr(12, 16, 1)
+    rp, col = to_dev(g)
+    root = int(np.argmax(g.degrees()))
+    with tq.BfsPlan(rp, col, capacity=64) as plan:
+        import torch
+        level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+        parent = torch.empty_like(level)
+        st = plan.run(root, level, parent, grow_on_full=True)
+        assert plan.regrows >= 1
+        check_against_oracle(g, root, level, parent, st)
+
+
 def test_plan_reuse_after_abort_and_many_runs(tq):
     import torch
     from inputs import kronecker_edges
