@@ -134,7 +134,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                 if (active) eok = bench_publish(q, et, item);
             } else if constexpr (VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
                 if (active) {
-                    et = tq_atom_add(q.rear, 1ull);
+                    et = tq_atom_add(per_lane_addr(q.rear), 1ull);
                     ++atom;
                     eok = bench_publish(q, et, item);
                 }
@@ -193,7 +193,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                 if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
                     dt = tq_warp_dequeue_n(q, active, &atom);
                 } else if (active) {
-                    dt = tq_atom_add(q.front, 1ull);
+                    dt = tq_atom_add(per_lane_addr(q.front), 1ull);
                     ++atom;
                 }
                 unsigned spins = 0;

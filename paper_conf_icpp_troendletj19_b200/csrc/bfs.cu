@@ -317,7 +317,7 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
         const unsigned mine = lane < cnt ? (cnt - lane + 31) / 32 : 0;
         unsigned long long base = 0;
         if (mine) {
-            base = tq_atom_add(q.rear, mine);
+            base = tq_atom_add(per_lane_addr(q.rear), mine);
             ++*qatom;
         }
         tq_fence_gpu();
@@ -348,7 +348,7 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
             const unsigned mine = lane < n ? (n - lane + 31) / 32 : 0;
             base = 0;
             if (mine) {
-                base = tq_atom_add(q.rear, mine);
+                base = tq_atom_add(per_lane_addr(q.rear), mine);
                 ++*qatom;
             }
             for (unsigned k = 0; k < mine; ++k)
@@ -451,7 +451,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     }
                 }
             } else if (!have) {
-                tk = (unsigned)tq_atom_add(q.front, 1ull);
+                tk = (unsigned)tq_atom_add(per_lane_addr(q.front), 1ull);
                 have = true;
                 ++st_qatom;
             }

@@ -16,6 +16,19 @@ namespace tqk {
 // of a task into "a fixed number of uniformly complex sub-tasks".
 constexpr uint32_t CHUNK_FLAG = 0x80000000u;
 
+// The per-thread-AFA comparator must issue one atomic per lane.  ptxas
+// warp-aggregates an atom.add whose address it can prove warp-uniform
+// (VOTEU.ANY + FLO + UPOPC + a single ATOMG: the paper's proxy lane, P:167,
+// inserted by the compiler).  Offsetting the address by (lane & zero), with
+// `zero` a device global that is always 0 but opaque to the compiler, keeps
+// the comparator's atomics per lane (checked in the SASS: one ATOMG per lane).
+static __device__ unsigned g_opaque_zero = 0;
+__device__ __forceinline__ unsigned long long *per_lane_addr(unsigned long long *p)
+{
+    const unsigned zero = *(volatile const unsigned *)&g_opaque_zero;
+    return p + (tq_lane() & zero);
+}
+
 constexpr int kStatCount = 16;
 enum StatIndex {
     ST_TASKS = 0,

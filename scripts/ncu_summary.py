@@ -23,18 +23,18 @@ def main(path):
     for k in KEYS:
         if k in d:
             print(f"{k:70s} {d[k][0]:>20s} {d[k][1]}")
-    stalls = [(h, v) for h, (v, u) in d.items()
-              if h.startswith("smsp__average_warp_latency_issue_stalled_") and h.endswith("_ratio") is False]
     st = []
+    pre = "smsp__pcsamp_warps_issue_stalled_"
     for h, (v, u) in d.items():
-        if h.startswith("smsp__warp_issue_stalled_") and h.endswith("_per_warp_active.pct"):
+        if h.startswith(pre) and not h.endswith("_not_issued"):
             try:
-                st.append((float(v), h))
+                st.append((float(v.replace(",", "")), h[len(pre):]))
             except ValueError:
                 pass
-    print("--- stall reasons (% of warp-active cycles) ---")
-    for v, h in sorted(st, reverse=True)[:12]:
-        print(f"{h[len('smsp__warp_issue_stalled_'):-len('_per_warp_active.pct')]:40s} {v:8.2f}")
+    tot = sum(v for v, _ in st) or 1.0
+    print("--- warp stall reasons (share of PC samples) ---")
+    for v, h in sorted(st, reverse=True)[:10]:
+        print(f"{h:40s} {100.0 * v / tot:7.2f}%")
 
 
 if __name__ == "__main__":
