@@ -173,6 +173,8 @@ typedef struct {
     uint64_t cas_failures;      /* CAS variants only                           */
     uint64_t empty_polls;       /* work cycles that found no data              */
     uint64_t tickets;           /* tasks enqueued (Rear advance)               */
+    uint64_t busy_cycles;       /* warp work cycles that processed >= 1 token  */
+    uint64_t rounds;            /* 128-edge expansion rounds                   */
     uint64_t skipped_tasks;     /* vertex tokens dropped by the expanded-level
                                    marker (already expanded at <= level)      */
     int32_t max_level;

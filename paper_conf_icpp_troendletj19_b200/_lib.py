@@ -46,7 +46,8 @@ class bfs_stats(ctypes.Structure):
                 ("tasks", c_u64), ("chunk_tasks", c_u64), ("edges_scanned", c_u64),
                 ("min_atomics", c_u64), ("reenqueues", c_u64), ("queue_atomics", c_u64),
                 ("cas_failures", c_u64), ("empty_polls", c_u64), ("tickets", c_u64),
-                ("skipped_tasks", c_u64), ("max_level", c_i32), ("persistent_threads", c_i32)]
+                ("busy_cycles", c_u64), ("rounds", c_u64), ("skipped_tasks", c_u64),
+                ("max_level", c_i32), ("persistent_threads", c_i32)]
 
 
 class tq_bench_cfg(ctypes.Structure):

@@ -397,8 +397,7 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     bp.lvl8 = p->lvl8;
     bp.x8 = p->x8;
     bp.parent_rule = p->parent_rule;
-    bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;
-    bp.stats = p->stats;
+    bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;    bp.stats = p->stats;
     bp.n_vertices = p->n;
     bp.chunk = p->chunk;
     bp.backoff_ns = p->backoff_ns;
@@ -453,6 +452,8 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
         stats->max_level = (int32_t)h[ST_MAX_LEVEL];
         stats->tickets = (ctr[1] - t0) + (p->hub_queue ? ctr[3] - t1 : 0ull);
         stats->skipped_tasks = h[ST_SKIPPED];
+        stats->busy_cycles = h[ST_BUSY_CYCLES];
+        stats->rounds = h[ST_ROUNDS];
         stats->persistent_threads = p->blocks * p->block;
     }
     if (status == TQ_FINISHED) return TQ_OK;

@@ -443,23 +443,19 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     }
                     pend1_mask = 0;
                 }
-                if (q1_lane) {
-                    if (have1) {
-                        const unsigned long long sv = tq_ld_relaxed(q1.slots + (tk1 & q1.mask));
-                        got1 = (unsigned)sv == tk1 + 1u;
-                        item = (uint32_t)(sv >> 32);
-                    }
-                }
             } else if (!have) {
                 tk = (unsigned)tq_atom_add(per_lane_addr(q.front), 1ull);
                 have = true;
                 ++st_qatom;
             }
-            if (have && !got1) {  // Listing 2 lines 3-5: non-atomic arrival check
-                const unsigned long long sv = tq_ld_relaxed(q.slots + (tk & q.mask));
-                got = (unsigned)sv == tk + 1u;
-                item = (uint32_t)(sv >> 32);
-            }
+            // Listing 2 lines 3-5: non-atomic arrival checks; a chunk-queue
+            // lane issues both polls back to back and prefers the chunk
+            const unsigned long long sv0 = have ? tq_ld_relaxed(q.slots + (tk & q.mask)) : 0ull;
+            const unsigned long long sv1 =
+                (q1_lane && have1) ? tq_ld_relaxed(q1.slots + (tk1 & q1.mask)) : 0ull;
+            got1 = q1_lane && have1 && (unsigned)sv1 == tk1 + 1u;
+            got = !got1 && have && (unsigned)sv0 == tk + 1u;
+            item = (uint32_t)((got1 ? sv1 : sv0) >> 32);
         } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
             got = cas_dequeue_one(q, &item, &st_qatom, &st_fail);
         } else {  // AN: every lane is hungry each cycle (no held tickets)
@@ -481,7 +477,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             if (lane == 0) ++S[ST_EMPTY_POLLS];
             ++idle;
             if ((idle & 3) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
-            if ((idle & 15) == 0) {
+            // termination test: 1 warp in 8, every 16 idle cycles, so idle
+            // warps do not crowd the Rear / Done lines busy warps update
+            if ((idle & 15) == 0 && (warp_gid & 7) == 0) {
                 bool fin = false;
                 if (lane == 0) {
                     // Done is read before Rear (R6): done(t1) ==
@@ -589,6 +587,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 S[ST_CHUNK_TASKS] += __popc(chm);
                 S[ST_SKIPPED] += __popc(skm);
                 S[ST_EDGES] += (unsigned)total;
+                S[ST_BUSY_CYCLES] += 1;
+                S[ST_ROUNDS] += (unsigned)((total + 32 * KU - 1) / (32 * KU));
             }
         }
         unsigned cnt = 0;

@@ -40,6 +40,8 @@ enum StatIndex {
     ST_CAS_FAILURES,
     ST_EMPTY_POLLS,
     ST_SKIPPED,
+    ST_BUSY_CYCLES,  // work cycles that processed >= 1 token
+    ST_ROUNDS,       // 32 x 4-edge expansion rounds
     // filled by the unpack kernel
     ST_REACHED,
     ST_DEG_SUM,

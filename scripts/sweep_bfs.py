@@ -41,5 +41,9 @@ for var, ch, th, bo in itertools.product(args.variants.split(","), map(int, args
                           "scan_x": round(st["edges_scanned"] / max(ideal, 1), 3),
                           "reenq_frac": round(st["reenqueues"] / max(st["reached"], 1), 3),
                           "tasks": st["tasks"], "chunk_tasks": st["chunk_tasks"], "min_atomics": st["min_atomics"],
-                          "qatom": st["queue_atomics"], "empty": st["empty_polls"], "maxlev": st["max_level"]}), flush=True)
+                          "qatom": st["queue_atomics"], "empty": st["empty_polls"], "maxlev": st["max_level"],
+                          "tok_per_cycle": round(st["tasks"] / max(st["busy_cycles"], 1), 2),
+                          "rounds_per_cycle": round(st["rounds"] / max(st["busy_cycles"], 1), 2),
+                          "round_fill": round(st["edges_scanned"] / max(128 * st["rounds"], 1), 3),
+                          "skipped": st["skipped_tasks"]}), flush=True)
     plan.close()
