@@ -58,6 +58,17 @@ __device__ __forceinline__ void tq_red_add_release(unsigned long long *p, unsign
 {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void tq_red_add_relaxed(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+/* Release fence (sm_100a SASS: MEMBAR.ALL.GPU; unlike fence.acq_rel it does
+ * not also invalidate L1).  An acquire is cheaper as a load: ld.acquire.gpu
+ * is LDG.STRONG.GPU + CCTL.IVALL, with no membar. */
+__device__ __forceinline__ void tq_fence_release()
+{
+    asm volatile("fence.release.gpu;" ::: "memory");
+}
 __device__ __forceinline__ void tq_st_relaxed(unsigned long long *p, unsigned long long v)
 {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -169,14 +180,15 @@ __device__ __forceinline__ unsigned long long tq_warp_dequeue_n(const tq_device_
 /* next lap ("picks up its work token from its slot and replaces it   */
 /* with the sentinel").  Non-blocking; per lane.               */
 /* ---------------------------------------------------------------- */
-/* The arrival check alone (Listing 2 lines 3-5): true if the item for
- * `ticket` has arrived.  The caller takes it: tq_fence_gpu() (acquire), then
- * stores seq = ticket + C to the slot (the reset half of tq_take). */
+/* The arrival check alone (Listing 2 lines 3-5), an acquire load: true if
+ * the item for `ticket` has arrived, and then everything the producer wrote
+ * before publishing it is visible.  The caller takes it by storing
+ * seq = ticket + C to the slot (the reset half of tq_take). */
 __device__ __forceinline__ bool tq_poll(const tq_device_view &q, unsigned long long ticket,
                                         unsigned int *item)
 {
     if (ticket == TQ_NO_TICKET) return false;
-    const unsigned long long v = tq_ld_relaxed(q.slots + (ticket & q.mask));
+    const unsigned long long v = tq_ld_acquire(q.slots + (ticket & q.mask));
     if ((unsigned int)v != (unsigned int)(ticket + 1)) return false;
     *item = (unsigned int)(v >> 32);
     return true;
@@ -187,7 +199,7 @@ __device__ __forceinline__ bool tq_take(const tq_device_view &q, unsigned long l
 {
     if (ticket == TQ_NO_TICKET) return false;
     unsigned long long *s = q.slots + (ticket & q.mask);
-    const unsigned long long v = tq_ld_relaxed(s);
+    const unsigned long long v = tq_ld_acquire(s);
     if ((unsigned int)v != (unsigned int)(ticket + 1)) return false;
     *item = (unsigned int)(v >> 32);
     tq_st_relaxed(s, (unsigned long long)(unsigned int)(ticket + q.mask + 1));
@@ -202,7 +214,7 @@ __device__ __forceinline__ bool tq_take(const tq_device_view &q, unsigned long l
 /* tq_publish: per lane, write one item to its reserved ticket after  */
 /* checking the slot still holds the dna sentinel for that ticket;    */
 /* otherwise raise the queue-full abort (P:268 line 25).  The caller  */
-/* must have issued tq_fence_gpu() after producing the task state the */
+/* must have issued tq_fence_release() after producing the task state the */
 /* item refers to.                                                    */
 /* ---------------------------------------------------------------- */
 __device__ __forceinline__ unsigned long long tq_warp_reserve_rear(const tq_device_view &q,
@@ -250,7 +262,7 @@ __device__ __forceinline__ unsigned long long tq_warp_enqueue_n(const tq_device_
     }
     const unsigned total = __shfl_sync(TQ_FULL_MASK, incl, 31);
     const unsigned long long base = tq_warp_reserve_rear(q, total, atomics);
-    tq_fence_gpu();
+    tq_fence_release();
     const unsigned long long mine = base + (incl - n_mine);
     bool ok = true;
 #pragma unroll

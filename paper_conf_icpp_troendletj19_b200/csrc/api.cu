@@ -400,6 +400,7 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;    bp.stats = p->stats;
     bp.n_vertices = p->n;
     bp.chunk = p->chunk;
+    while ((1 << bp.log2_chunk) < p->chunk) ++bp.log2_chunk;
     bp.backoff_ns = p->backoff_ns;
     bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
 

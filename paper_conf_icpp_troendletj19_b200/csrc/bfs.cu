@@ -290,7 +290,9 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
         } else {
             if (!an_reserve_rear(q, cnt, &base, qatom, casfail)) return;
         }
-        if (!(flags & 2)) tq_fence_gpu();  // release: W updates before the tokens that name them
+        // release: the W updates (and this warp's Rear reservation) are
+        // ordered before the tokens that name them
+        if (!(flags & 2)) tq_fence_release();
         for (unsigned i0 = 0; i0 < cnt; i0 += 32 * 4) {
             unsigned long long sv[4];
 #pragma unroll
@@ -320,10 +322,10 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
             base = tq_atom_add(per_lane_addr(q.rear), mine);
             ++*qatom;
         }
-        tq_fence_gpu();
+        tq_fence_release();
         for (unsigned k = 0; k < mine; ++k) tq_publish(q, base + k, items[lane + 32 * k]);
     } else {  // CAS_RETRY: one CAS-reserved slot per item, per lane
-        tq_fence_gpu();
+        tq_fence_release();
         for (unsigned i = lane; i < cnt; i += 32)
             if (!cas_enqueue_one(q, items[i], qatom, casfail)) break;
     }
@@ -450,9 +452,11 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
             // Listing 2 lines 3-5: non-atomic arrival checks; a chunk-queue
             // lane issues both polls back to back and prefers the chunk
-            const unsigned long long sv0 = have ? tq_ld_relaxed(q.slots + (tk & q.mask)) : 0ull;
+            // (acquire loads: a hit makes the producer's W update visible,
+            // with no fence; ld.acquire.gpu is LDG.STRONG.GPU + CCTL.IVALL)
+            const unsigned long long sv0 = have ? tq_ld_acquire(q.slots + (tk & q.mask)) : 0ull;
             const unsigned long long sv1 =
-                (q1_lane && have1) ? tq_ld_relaxed(q1.slots + (tk1 & q1.mask)) : 0ull;
+                (q1_lane && have1) ? tq_ld_acquire(q1.slots + (tk1 & q1.mask)) : 0ull;
             got1 = q1_lane && have1 && (unsigned)sv1 == tk1 + 1u;
             got = !got1 && have && (unsigned)sv0 == tk + 1u;
             item = (uint32_t)((got1 ? sv1 : sv0) >> 32);
@@ -503,7 +507,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         backoff = 0;
         idle = 0;
         if (((++busy) & 63) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
-        if (!(p.exp_flags & 1)) tq_fence_gpu();  // acquire: the producer's W update is visible now
+        if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY || VARIANT == TQ_VARIANT_AN)
+            tq_fence_gpu();  // acquire for the comparators' relaxed dequeues
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
             if (got0) {  // put the slot back to dna for the next lap
                 tq_st_relaxed(q.slots + (tk & q.mask), (unsigned long long)(tk + cap32));
@@ -549,7 +554,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 lo = ld_nc_i64(p.row_ptr + v);
                 hi = ld_nc_i64(p.row_ptr + v + 1);
                 if (hi - lo > chunk) {  // hub: schedule its sub-tasks instead
-                    nch = (unsigned)((hi - lo + chunk - 1) / chunk);
+                    nch = (unsigned)((hi - lo + chunk - 1) >> p.log2_chunk);
                     chb = (uint32_t)p.hub_base[v];
                     hi = lo;
                 }
@@ -616,7 +621,13 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             // are never below the true level, R8)
             unsigned m8[KU];
 #pragma unroll
-            for (int j = 0; j < KU; ++j) m8[j] = val[j] ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : 0u;
+            for (int j = 0; j < KU; ++j) {
+                // offers at level >= 254 cannot be filtered by the saturated
+                // mirror: skip the probe (saves a dependent round trip on deep
+                // graphs, e.g. the grid's 8,191 levels) and go to atomicMin
+                const bool deep = (unsigned)(off[j] >> 32) >= kLvlSat;
+                m8[j] = (val[j] && !deep) ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : kLvlSat;
+            }
             bool cand[KU], tie[KU];
 #pragma unroll
             for (int j = 0; j < KU; ++j) {
@@ -678,6 +689,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.exp_flags);
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
+        const bool hubm_any = hubm != 0;
         while (hubm) {
             const int h = __ffs(hubm) - 1;
             hubm &= hubm - 1;
@@ -691,19 +703,22 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         // it is ordered after this warp's Rear reservations; idle warps
         // compare Done with Rear.
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
-            // lane 0 issued every Rear reservation of this warp
+            // lane 0 issued every Rear reservation of this warp.  The release
+            // fence before publishing staged tokens already ordered them; only
+            // a cycle that ended with chunk reservations (published without
+            // a fence) needs a release on Done itself.
             if (lane == 0) {
-                if (p.exp_flags & 4)
-                    atomicAdd(q.done, (unsigned long long)__popc(gm));
-                else
+                if (hubm_any)
                     tq_red_add_release(q.done, (unsigned long long)__popc(gm));
+                else
+                    tq_red_add_relaxed(q.done, (unsigned long long)__popc(gm));
                 ++st_qatom;
             }
         } else {
             __syncwarp();
-            tq_fence_gpu();
+            tq_fence_release();
             if (got) {
-                tq_red_add_release(q.done, 1ull);
+                tq_red_add_relaxed(q.done, 1ull);
                 ++st_qatom;
             }
         }

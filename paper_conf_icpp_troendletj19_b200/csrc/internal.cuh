@@ -64,6 +64,7 @@ struct BfsParams {
     unsigned long long *stats; // kStatCount counters
     int64_t n_vertices;
     int chunk;                 // max edges per token (power of 2)
+    int log2_chunk;
     int backoff_ns;            // max idle back-off, 0 = none
     int parent_rule;           // TQ_PARENT_ANY / TQ_PARENT_MIN_ID (include/tq.h)
     unsigned exp_flags;        // experiments only (TQ_EXP_FLAGS env), 0 in production
