@@ -204,6 +204,13 @@ tq_status bfs_plan_create(const tq_csr *g, const bfs_opts *opts, bfs_plan **out)
  * opts->stream, but synchronous (it reads the status word back). */
 tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,
                        bfs_stats *stats);
+/* Asynchronous form: bfs_plan_launch enqueues the run on the plan's stream
+ * and returns; bfs_plan_wait blocks until it finished and returns its status
+ * (and statistics).  At most one run per plan in flight (TQ_ERR_INVALID
+ * otherwise); outputs must be device pointers.  Several plans on different
+ * streams run concurrently (multi-root batches). */
+tq_status bfs_plan_launch(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out);
+tq_status bfs_plan_wait(bfs_plan *p, bfs_stats *stats);
 tq_status bfs_plan_destroy(bfs_plan *p);
 
 /* ------------------------------------------------------------------------ */

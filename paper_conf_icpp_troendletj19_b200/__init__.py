@@ -5,7 +5,7 @@ Workloads on GPUs", ICPP 2019. The product is `libtq.so` (CUDA for sm_100a
 behind the C ABI in include/tq.h); this package is its thin Python binding.
 """
 from .api import (BfsPlan, Queue, TQError, VARIANTS, bfs, persistent_threads, queue_bench,
-                  version)
+                  run_concurrent, version)
 
 __all__ = ["BfsPlan", "Queue", "TQError", "VARIANTS", "bfs", "persistent_threads", "queue_bench",
-           "version"]
+           "run_concurrent", "version"]

@@ -161,6 +161,16 @@ class BfsPlan:
             check(status, "bfs_plan_run")
             return _stats_dict(st)
 
+    def launch(self, root: int, level=None, parent=None):
+        """Enqueue one BFS on the plan's stream and return (bfs_plan_launch)."""
+        check(lib().bfs_plan_launch(self._h, int(root), _ptr(level), _ptr(parent)), "bfs_plan_launch")
+
+    def wait(self) -> dict:
+        """Block until the launched BFS finished; its statistics (bfs_plan_wait)."""
+        st = _lib.bfs_stats()
+        check(lib().bfs_plan_wait(self._h, ctypes.byref(st)), "bfs_plan_wait")
+        return _stats_dict(st)
+
     def close(self):
         h = getattr(self, "_h", None)
         if h is not None and h.value:
@@ -178,6 +188,25 @@ class BfsPlan:
 
     def __exit__(self, *a):
         self.close()
+
+
+def run_concurrent(plans, roots, levels=None, parents=None):
+    """Run `roots` over several plans (each on its own stream) keeping one BFS
+    in flight per plan; returns the per-root statistics in root order."""
+    out = [None] * len(roots)
+    busy = {}  # plan index -> root index
+    nxt = 0
+    k = len(plans)
+    while nxt < len(roots) or busy:
+        for i in range(k):
+            if i not in busy and nxt < len(roots):
+                plans[i].launch(roots[nxt], levels[i] if levels else None, parents[i] if parents else None)
+                busy[i] = nxt
+                nxt += 1
+        # wait for the oldest launch first (launch order == root order)
+        i = min(busy, key=busy.get)
+        out[busy.pop(i)] = plans[i].wait()
+    return out
 
 
 class Queue:

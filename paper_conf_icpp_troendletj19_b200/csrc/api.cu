@@ -115,6 +115,11 @@ struct bfs_plan {
     unsigned long long next_ticket1 = 0;
     unsigned long long *stats = nullptr;      // device, kStatCount
     unsigned long long *stats_h = nullptr;    // pinned
+    unsigned long long *ctr_h = nullptr;      // pinned: front, rear, done, rear1, status
+    bool in_flight = false;                   // launched, not yet waited for
+    size_t l2_window = 0;                     // persisting-L2 window over lvl8
+    size_t l2_limit_saved = 0;                // device persisting-L2 limit to restore
+    bool l2_limit_set = false;
     unsigned long long next_ticket = 0;
     bool dirty = false;
     int32_t *out_scratch = nullptr;           // for host outputs
@@ -257,6 +262,9 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     cudaFree(p->stats);
     cudaFree(p->out_scratch);
     if (p->stats_h) cudaFreeHost(p->stats_h);
+    if (p->ctr_h) cudaFreeHost(p->ctr_h);
+    if (p->l2_window) cudaCtxResetPersistingL2Cache();
+    if (p->l2_limit_set) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, p->l2_limit_saved);
     tq_destroy(p->q);
     tq_destroy(p->q1);
     delete p;
@@ -328,6 +336,7 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (e == cudaSuccess) e = cudaMalloc(&p->x8, (size_t)n);
     if (e == cudaSuccess) e = cudaMalloc(&p->stats, kStatCount * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMallocHost(&p->ctr_h, 8 * sizeof(unsigned long long));
     for (auto &ev : p->ev)
         if (e == cudaSuccess) e = cudaEventCreate(&ev);
     if (e != cudaSuccess) return fail(from_cuda(e));
@@ -361,16 +370,39 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
         p->blocks = full;
     }
     if (p->blocks < 1) p->blocks = 1;
+    {
+        // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the byte
+        // mirror is probed once per edge; a persisting window keeps it
+        // resident against the col stream.  The device-wide carve-out is
+        // raised here if needed and restored by bfs_plan_destroy.
+        int max_win = 0, max_persist = 0;
+        cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, gdev);
+        cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, gdev);
+        size_t w = (size_t)n;
+        if (w > (size_t)max_win) w = (size_t)max_win;
+        if (w > (size_t)max_persist) w = (size_t)max_persist;
+        size_t cur = 0;
+        if (w > 0 && cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
+            if (cur < w && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, w) == cudaSuccess) {
+                p->l2_limit_saved = cur;
+                p->l2_limit_set = true;
+            }
+            p->l2_window = w;
+        }
+        cudaGetLastError();
+    }
     e = cudaStreamSynchronize(p->stream);
     if (e != cudaSuccess) return fail(from_cuda(e));
     *out = p;
     return TQ_OK;
 }
 
-static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int32_t *parent,
-                                 bfs_stats *stats)
+// First half of a run: enqueue init + persistent kernel + unpack and the
+// status / statistics read-back on the plan's stream; returns immediately.
+static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t *parent)
 {
     cudaStream_t s = p->stream;
+    if (p->in_flight) return TQ_ERR_INVALID;
     if (p->dirty) {
         tq_status st = tq_reset(p->q, s);
         if (st == TQ_OK && p->q1) st = tq_reset(p->q1, s);
@@ -397,12 +429,14 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     bp.lvl8 = p->lvl8;
     bp.x8 = p->x8;
     bp.parent_rule = p->parent_rule;
-    bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;    bp.stats = p->stats;
+    bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;
+    bp.stats = p->stats;
     bp.n_vertices = p->n;
     bp.chunk = p->chunk;
     while ((1 << bp.log2_chunk) < p->chunk) ++bp.log2_chunk;
     bp.backoff_ns = p->backoff_ns;
     bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
+    bp.l2_window_bytes = (bp.exp_flags & 32) ? 0 : p->l2_window;
 
     CK(cudaEventRecord(p->ev[0], s));
     CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));
@@ -413,15 +447,26 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     CK(cudaEventRecord(p->ev[3], s));
     CK(cudaMemcpyAsync(p->stats_h, p->stats, kStatCount * sizeof(unsigned long long),
                        cudaMemcpyDeviceToHost, s));
-    unsigned long long ctr[4] = {0, 0, 0, 0};
-    unsigned status = 0;
+    unsigned long long *ctr = p->ctr_h;  // pinned: front, rear, done, rear1, status
+    ctr[3] = 0;
     CK(cudaMemcpyAsync(&ctr[0], p->q->view.front, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&ctr[1], p->q->view.rear, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&ctr[2], p->q->view.done, 8, cudaMemcpyDeviceToHost, s));
     if (p->hub_queue) CK(cudaMemcpyAsync(&ctr[3], p->q1->view.rear, 8, cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(&status, p->q->view.status, 4, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
+    CK(cudaMemcpyAsync(&ctr[4], p->q->view.status, 4, cudaMemcpyDeviceToHost, s));
+    p->in_flight = true;
+    return TQ_OK;
+}
 
+// Second half of a run: wait for the launch, read the status word back and
+// fill the statistics.
+static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
+{
+    if (!p->in_flight) return TQ_ERR_INVALID;
+    p->in_flight = false;
+    CK(cudaStreamSynchronize(p->stream));
+    const unsigned long long *ctr = p->ctr_h;
+    const unsigned status = (unsigned)ctr[4];
     const unsigned long long t0 = p->next_ticket, t1 = p->next_ticket1;
     if (status == TQ_FINISHED) {
         // every reserved ticket below Rear was taken; slots of tickets
@@ -463,6 +508,23 @@ static tq_status plan_run_device(bfs_plan *p, int32_t root, int32_t *level, int3
     return TQ_ERR_CUDA;
 }
 
+tq_status bfs_plan_launch(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out)
+{
+    if (!p || root < 0 || root >= p->n) return TQ_ERR_INVALID;
+    if ((level_out && !is_device_ptr(level_out, nullptr)) ||
+        (parent_out && !is_device_ptr(parent_out, nullptr)))
+        return TQ_ERR_INVALID;  // the asynchronous form takes device outputs only
+    DeviceGuard g(p->device);
+    return plan_launch(p, root, level_out, parent_out);
+}
+
+tq_status bfs_plan_wait(bfs_plan *p, bfs_stats *stats)
+{
+    if (!p) return TQ_ERR_INVALID;
+    DeviceGuard g(p->device);
+    return plan_finish(p, stats);
+}
+
 tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,
                        bfs_stats *stats)
 {
@@ -470,11 +532,15 @@ tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *p
     DeviceGuard g(p->device);
     const bool host_l = level_out && !is_device_ptr(level_out, nullptr);
     const bool host_p = parent_out && !is_device_ptr(parent_out, nullptr);
-    if (!host_l && !host_p) return plan_run_device(p, root, level_out, parent_out, stats);
+    if (!host_l && !host_p) {
+        const tq_status st = plan_launch(p, root, level_out, parent_out);
+        return st == TQ_OK ? plan_finish(p, stats) : st;
+    }
     if (!p->out_scratch) CK(cudaMalloc(&p->out_scratch, (size_t)p->n * 2 * sizeof(int32_t)));
     int32_t *dl = level_out ? (host_l ? p->out_scratch : level_out) : nullptr;
     int32_t *dp = parent_out ? (host_p ? p->out_scratch + p->n : parent_out) : nullptr;
-    tq_status st = plan_run_device(p, root, dl, dp, stats);
+    tq_status st = plan_launch(p, root, dl, dp);
+    if (st == TQ_OK) st = plan_finish(p, stats);
     if (st != TQ_OK) return st;
     if (host_l)
         CK(cudaMemcpyAsync(level_out, dl, (size_t)p->n * sizeof(int32_t), cudaMemcpyDeviceToHost, p->stream));

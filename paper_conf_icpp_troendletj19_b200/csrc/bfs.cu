@@ -898,8 +898,25 @@ template <int V, int KU = kU, int MINB = kMinBlocks>
 static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStream_t s)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
-    bfs_persistent_kernel<V, KU, MINB><<<blocks, kBlock, 0, s>>>(p);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(blocks);
+    cfg.blockDim = dim3(kBlock);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    if (p.l2_window_bytes) {
+        // keep the byte level mirror (probed once per edge) resident in the
+        // persisting part of L2 while the col stream and the per-task arrays
+        // pass through
+        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[0].val.accessPolicyWindow.base_ptr = (void *)p.lvl8;
+        attr[0].val.accessPolicyWindow.num_bytes = p.l2_window_bytes;
+        attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
+        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+    }
+    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, KU, MINB>, p);
 }
 
 // tuning instances (TQ_EXP_FLAGS >> 8): resident blocks per SM

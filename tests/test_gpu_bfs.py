@@ -170,6 +170,33 @@ def test_queue_full_aborts_and_retry_succeeds(tq):
     check_against_oracle(g, root, level, parent, st)
 
 
+def test_concurrent_plans_on_two_streams(tq):
+    """bfs_plan_launch / bfs_plan_wait: two BFS in flight at once on two
+    streams (half the persistent grid each); both results exact."""
+    import torch
+    g = kronecker_csr(13, 16, 3)
+    rp, col = to_dev(g)
+    half = tq.persistent_threads() // 2
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    plans = [tq.BfsPlan(rp, col, stream=s, threads=half, parents=pr) for s, pr in zip(streams, ["any", "min_id"])]
+    lv = [torch.empty(g.n_vertices, dtype=torch.int32, device="cuda") for _ in plans]
+    pa = [torch.empty_like(lv[0]) for _ in plans]
+    roots = [int(r) for r in sample_roots(g.row_ptr, 6, 8)]
+    for k in range(0, len(roots), 2):
+        for i in range(2):
+            plans[i].launch(roots[k + i], lv[i], pa[i])
+        for i in range(2):
+            st = plans[i].wait()
+            check_against_oracle(g, roots[k + i], lv[i], pa[i], st, min_id=(i == 1))
+    with pytest.raises(tq.TQError):
+        plans[0].wait()  # nothing in flight
+    stats = tq.run_concurrent(plans, roots)
+    assert [s["reached"] for s in stats] == [oracle.bfs(g.row_ptr, g.col, r, parents=False)[2]["reached"]
+                                             for r in roots]
+    for p_ in plans:
+        p_.close()
+
+
 def test_grow_on_full_retries_with_larger_queue(tq):
     g = kronecker_csr(12, 16, 1)
     rp, col = to_dev(g)
