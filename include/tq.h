@@ -55,8 +55,12 @@ typedef enum {
                                       and on empty            */
     TQ_VARIANT_AN = 3,             /* AN: BASE + arbitrary-n (proxy CAS loop
                                       reserving n slots)             */
-    TQ_VARIANT_ATOMIC_CEILING = 4  /* tq_bench only: proxy atomicAdd on Rear
+    TQ_VARIANT_ATOMIC_CEILING = 4, /* tq_bench only: proxy atomicAdd on Rear
                                       with no slot traffic -> R_atom          */
+    TQ_VARIANT_RF_AN_CTA = 5       /* tq_bench only: RF/AN with the CTA as the
+                                      proxy group (one atomicAdd on Rear and
+                                      one on Front per block per iteration;
+                                      the abstract's "thread group")   */
 } tq_variant;
 
 /* ------------------------------------------------------------------------ */

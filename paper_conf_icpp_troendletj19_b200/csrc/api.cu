@@ -574,7 +574,7 @@ tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
 {
     if (!c || !r) return TQ_ERR_INVALID;
     memset(r, 0, sizeof(*r));
-    if (c->variant < TQ_VARIANT_RF_AN || c->variant > TQ_VARIANT_ATOMIC_CEILING) return TQ_ERR_UNSUPPORTED;
+    if (c->variant < TQ_VARIANT_RF_AN || c->variant > TQ_VARIANT_RF_AN_CTA) return TQ_ERR_UNSUPPORTED;
     if (c->batch < 1 || c->batch > 32 || c->items == 0 || c->warps < 0) return TQ_ERR_INVALID;
     DeviceGuard g(c->device);
     if (!g.ok) return TQ_ERR_INVALID;

@@ -109,12 +109,68 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
     unsigned long long s_enq = 0, s_deq = 0, x_enq = 0, x_deq = 0, sink = 0;
     const unsigned long long deadline = tq_globaltimer() + p.timeout_ns;
     bool stop = false;
+    // RF_AN_CTA: the proxy group is the whole CTA (double-buffered bases)
+    __shared__ unsigned long long cta_base[2][2];
+    const unsigned wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
 
-    for (int it = 0; it < p.iters && !stop; ++it) {
+    // (the CTA variant leaves the loop only through its block-wide vote)
+    for (int it = 0; it < p.iters && (VARIANT == TQ_VARIANT_RF_AN_CTA || !stop); ++it) {
         const unsigned long long g = (warp_gid * (unsigned long long)p.iters + it) * p.batch + lane;
         const uint32_t item = item_of(p.seed32, g);
 
-        if constexpr (VARIANT == TQ_VARIANT_ATOMIC_CEILING) {
+        if constexpr (VARIANT == TQ_VARIANT_RF_AN_CTA) {
+            // One thread reserves the enqueue tickets and the dequeue tickets
+            // of all warps of the block (arbitrary-n with a CTA-wide proxy
+            // group, "a proxy thread in each thread group"); warp w owns
+            // [base + w*b, base + (w+1)*b) of each.
+            unsigned long long *cb = cta_base[it & 1];
+            if (threadIdx.x == 0) {
+                const unsigned long long n = (unsigned long long)nwb * p.batch;
+                cb[0] = tq_atom_add(q.rear, n);
+                cb[1] = tq_atom_add(q.front, n);
+                atom += 2;
+            }
+            if (__syncthreads_or(stop)) break;
+            const unsigned long long et = cb[0] + (unsigned long long)wib * p.batch + lane;
+            const unsigned long long dt = cb[1] + (unsigned long long)wib * p.batch + lane;
+            bool eok = true;
+            if (active) {
+                eok = bench_publish(q, et, item);
+                if (eok) {
+                    ++n_enq;
+                    const unsigned long long f = mix64(item);
+                    s_enq += f;
+                    x_enq ^= f;
+                    if (p.enq_log) p.enq_log[et] = item;
+                }
+            }
+            if (active && eok) {
+                uint32_t got_item = 0;
+                unsigned spins = 0;
+                bool have = false;
+                while (!have) {
+                    have = tq_take(q, dt, &got_item);
+                    if (!have && (++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {
+                        stop = true;
+                        break;
+                    }
+                    if (!have) ++empty;
+                }
+                if (have) {
+                    ++n_deq;
+                    const unsigned long long f = mix64(got_item);
+                    s_deq += f;
+                    x_deq ^= f;
+                    if (p.deq_log) p.deq_log[dt] = got_item;
+                    uint32_t x = got_item;
+                    for (int w = 0; w < p.work_iters; ++w) x = x * 1664525u + 1013904223u;
+                    sink += x;
+                }
+            } else if (active) {
+                stop = true;
+            }
+            continue;
+        } else if constexpr (VARIANT == TQ_VARIANT_ATOMIC_CEILING) {
             if (lane == 0) {
                 sink += tq_atom_add(q.rear, (unsigned long long)p.batch);
                 ++atom;
@@ -316,6 +372,7 @@ cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int bloc
     case TQ_VARIANT_CAS_RETRY: return launch_b<TQ_VARIANT_CAS_RETRY>(p, blocks, block, s);
     case TQ_VARIANT_AN: return launch_b<TQ_VARIANT_AN>(p, blocks, block, s);
     case TQ_VARIANT_ATOMIC_CEILING: return launch_b<TQ_VARIANT_ATOMIC_CEILING>(p, blocks, block, s);
+    case TQ_VARIANT_RF_AN_CTA: return launch_b<TQ_VARIANT_RF_AN_CTA>(p, blocks, block, s);
     default: return cudaErrorInvalidValue;
     }
 }
@@ -333,6 +390,8 @@ cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm)
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_AN>, block, 0);
     case TQ_VARIANT_ATOMIC_CEILING:
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_ATOMIC_CEILING>, block, 0);
+    case TQ_VARIANT_RF_AN_CTA:
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_kernel<TQ_VARIANT_RF_AN_CTA>, block, 0);
     default: return cudaErrorInvalidValue;
     }
 }

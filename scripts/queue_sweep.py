@@ -20,7 +20,7 @@ from inputs import fingerprint, item_of
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--out", default="gpurun_out/queue_sweep.jsonl")
-ap.add_argument("--variants", default="rf_an,per_thread_afa,cas_retry,an,atomic_ceiling")
+ap.add_argument("--variants", default="rf_an,rf_an_cta,per_thread_afa,cas_retry,an,atomic_ceiling")
 ap.add_argument("--batches", default="1,2,4,8,16,32")
 ap.add_argument("--capacity", type=int, default=1 << 20)
 ap.add_argument("--big-capacity", type=int, default=1 << 26)

@@ -10,7 +10,7 @@ from inputs import fingerprint, item_of
 
 pytestmark = pytest.mark.gpu
 
-VARIANTS = ["rf_an", "per_thread_afa", "cas_retry", "an"]
+VARIANTS = ["rf_an", "per_thread_afa", "cas_retry", "an", "rf_an_cta"]
 
 
 @pytest.fixture(scope="module")
