@@ -429,14 +429,13 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.lvl8 = p->lvl8;
     bp.x8 = p->x8;
     bp.parent_rule = p->parent_rule;
-    bp.exp_flags = getenv("TQ_EXP_FLAGS") ? (unsigned)atoi(getenv("TQ_EXP_FLAGS")) : 0u;
     bp.stats = p->stats;
     bp.n_vertices = p->n;
     bp.chunk = p->chunk;
     while ((1 << bp.log2_chunk) < p->chunk) ++bp.log2_chunk;
     bp.backoff_ns = p->backoff_ns;
     bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
-    bp.l2_window_bytes = (bp.exp_flags & 32) ? 0 : p->l2_window;
+    bp.l2_window_bytes = p->l2_window;
 
     CK(cudaEventRecord(p->ev[0], s));
     CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));

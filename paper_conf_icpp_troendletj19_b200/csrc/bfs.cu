@@ -280,7 +280,7 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const uint32_t *items,
                                                unsigned cnt, unsigned lane, unsigned *qatom,
-                                               unsigned *casfail, unsigned flags = 0)
+                                               unsigned *casfail)
 {
     if (cnt == 0) return;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
@@ -292,7 +292,7 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
         }
         // release: the W updates (and this warp's Rear reservation) are
         // ordered before the tokens that name them
-        if (!(flags & 2)) tq_fence_release();
+        tq_fence_release();
         for (unsigned i0 = 0; i0 < cnt; i0 += 32 * 4) {
             unsigned long long sv[4];
 #pragma unroll
@@ -678,7 +678,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
             if (cnt > kStageCap - 32 * KU) {
                 __syncwarp();
-                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.exp_flags);
+                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
                 __syncwarp();
                 cnt = 0;
             }
@@ -686,7 +686,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
-        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.exp_flags);
+        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
         const bool hubm_any = hubm != 0;
@@ -919,21 +919,9 @@ static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStrea
     return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, KU, MINB>, p);
 }
 
-// tuning instances (TQ_EXP_FLAGS >> 8): resident blocks per SM
-#define TQ_EXP_INSTANCES(X) X(1, 4, 4) X(2, 4, 5) X(3, 4, 7) X(4, 4, 8)
-
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
                                   cudaStream_t s)
 {
-    if (variant == TQ_VARIANT_RF_AN && (p.exp_flags >> 8)) {
-        switch (p.exp_flags >> 8) {
-#define X(id, ku, mb) \
-    case id: return launch_v<TQ_VARIANT_RF_AN, ku, mb>(p, blocks, block, s);
-            TQ_EXP_INSTANCES(X)
-#undef X
-        default: return cudaErrorInvalidValue;
-        }
-    }
     switch (variant) {
     case TQ_VARIANT_RF_AN: return launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
     case TQ_VARIANT_PER_THREAD_AFA: return launch_v<TQ_VARIANT_PER_THREAD_AFA>(p, blocks, block, s);
@@ -946,19 +934,6 @@ cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, i
 cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
-    const char *ef = getenv("TQ_EXP_FLAGS");
-    const unsigned exp = ef ? (unsigned)atoi(ef) >> 8 : 0u;
-    if (variant == TQ_VARIANT_RF_AN && exp) {
-        switch (exp) {
-#define X(id, ku, mb)                                              \
-    case id:                                                       \
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(      \
-            blocks_per_sm, bfs_persistent_kernel<TQ_VARIANT_RF_AN, ku, mb>, kBlock, 0);
-            TQ_EXP_INSTANCES(X)
-#undef X
-        default: return cudaErrorInvalidValue;
-        }
-    }
     switch (variant) {
     case TQ_VARIANT_RF_AN:
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(

@@ -67,7 +67,6 @@ struct BfsParams {
     int log2_chunk;
     int backoff_ns;            // max idle back-off, 0 = none
     int parent_rule;           // TQ_PARENT_ANY / TQ_PARENT_MIN_ID (include/tq.h)
-    unsigned exp_flags;        // experiments only (TQ_EXP_FLAGS env), 0 in production
     unsigned long long timeout_ns;
     size_t l2_window_bytes;    // persisting-L2 window over lvl8 (0 = none)
 };

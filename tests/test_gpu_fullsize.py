@@ -74,6 +74,29 @@ def test_kron26_levels_identical(tq):
     _kron_check(tq, 26, 1)
 
 
+@pytest.mark.parametrize("variant", ["rf_an", "per_thread_afa", "an"])
+def test_paper_synthetic_tree_closed_form(tq, variant):
+    """P:301 synthetic dataset (reading R13): 10,485,760-vertex heap-ordered
+    4-ary tree; level(i) = k iff 4^k <= 3i+1 < 4^(k+1), parent (i-1)/4."""
+    import torch
+    import inputs.gpu as gg
+    n = 10485760
+    rp, col = gg.tree4_csr_cuda(n)
+    level, parent, st = tq.bfs(rp, col, 0, variant=variant, parents="min_id", timeout_s=60)
+    i = torch.arange(n, device="cuda", dtype=torch.int64)
+    x = 3 * i + 1
+    exp = torch.zeros(n, dtype=torch.int64, device="cuda")
+    k, p4 = 0, 1
+    while p4 * 4 <= int(x.max()):
+        k += 1
+        p4 *= 4
+        exp[x >= p4] = k
+    assert torch.equal(level.long(), exp)
+    exp_par = torch.where(i > 0, (i - 1) // 4, torch.zeros_like(i))
+    assert torch.equal(parent.long(), exp_par)
+    assert st["traversed_edges"] == n - 1
+
+
 def test_queue_bench_full_size_conserves(tq):
     from inputs import fingerprint, item_of
     for variant in ("rf_an", "per_thread_afa", "cas_retry", "an"):
