@@ -215,6 +215,15 @@ tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *p
  * streams run concurrently (multi-root batches). */
 tq_status bfs_plan_launch(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out);
 tq_status bfs_plan_wait(bfs_plan *p, bfs_stats *stats);
+/* A batch of roots.  Root i writes level_out + i * out_stride and
+ * parent_out + i * out_stride (host or device; either may be NULL;
+ * out_stride = 0 reuses one buffer, leaving the last root's result).  Host
+ * outputs are copied from double-buffered device scratch on a second stream,
+ * overlapped with the next root's BFS.  stats: NULL or n_roots entries.
+ * Synchronous; stops at the first non-OK root and returns its status. */
+tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
+                             int32_t *level_out, int32_t *parent_out, int64_t out_stride,
+                             bfs_stats *stats);
 tq_status bfs_plan_destroy(bfs_plan *p);
 
 /* ------------------------------------------------------------------------ */

@@ -80,6 +80,7 @@ EXPORTS = {
     "bfs_plan_destroy": (ctypes.c_int, [c_vp]),
     "bfs_plan_launch": (ctypes.c_int, [c_vp, c_i32, c_vp, c_vp]),
     "bfs_plan_wait": (ctypes.c_int, [c_vp, ctypes.POINTER(bfs_stats)]),
+    "bfs_plan_run_batch": (ctypes.c_int, [c_vp, c_vp, c_i32, c_vp, c_vp, c_i64, c_vp]),
     "tq_bench": (ctypes.c_int, [ctypes.POINTER(tq_bench_cfg), ctypes.POINTER(tq_bench_result)]),
     "tq_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "tq_persistent_threads": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int,

@@ -161,6 +161,21 @@ class BfsPlan:
             check(status, "bfs_plan_run")
             return _stats_dict(st)
 
+    def run_batch(self, roots, level=None, parent=None, stride: int | None = None) -> list:
+        """`bfs_plan_run_batch`: root i writes level[i * stride:] / parent[...].
+        stride defaults to n_vertices when the outputs hold len(roots) rows,
+        else 0 (one reused buffer). Host outputs are copied on a second stream
+        overlapped with the next BFS. Returns the per-root statistics."""
+        r = np.ascontiguousarray(np.asarray(roots, dtype=np.int32))
+        n = r.size
+        if stride is None:
+            size = level.shape[0] if level is not None else (parent.shape[0] if parent is not None else 0)
+            stride = self.n_vertices if size >= n * self.n_vertices and n > 1 else 0
+        sts = (_lib.bfs_stats * max(n, 1))()
+        check(lib().bfs_plan_run_batch(self._h, r.ctypes.data, n, _ptr(level), _ptr(parent), int(stride),
+                                       ctypes.cast(sts, ctypes.c_void_p)), "bfs_plan_run_batch")
+        return [_stats_dict(sts[i]) for i in range(n)]
+
     def launch(self, root: int, level=None, parent=None):
         """Enqueue one BFS on the plan's stream and return (bfs_plan_launch)."""
         check(lib().bfs_plan_launch(self._h, int(root), _ptr(level), _ptr(parent)), "bfs_plan_launch")

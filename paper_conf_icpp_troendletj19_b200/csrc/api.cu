@@ -117,6 +117,9 @@ struct bfs_plan {
     unsigned long long *stats_h = nullptr;    // pinned
     unsigned long long *ctr_h = nullptr;      // pinned: front, rear, done, rear1, status
     bool in_flight = false;                   // launched, not yet waited for
+    int32_t *dbuf[2] = {nullptr, nullptr};    // batch: double-buffered device outputs
+    cudaStream_t copy_stream = nullptr;       // batch: D2H copies
+    cudaEvent_t bfs_done[2] = {nullptr, nullptr}, copy_done[2] = {nullptr, nullptr};
     size_t l2_window = 0;                     // persisting-L2 window over lvl8
     size_t l2_limit_saved = 0;                // device persisting-L2 limit to restore
     bool l2_limit_set = false;
@@ -261,6 +264,13 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     cudaFree(p->chunk_tab);
     cudaFree(p->stats);
     cudaFree(p->out_scratch);
+    if (p->copy_stream) cudaStreamSynchronize(p->copy_stream);
+    for (int b = 0; b < 2; ++b) {
+        cudaFree(p->dbuf[b]);
+        if (p->bfs_done[b]) cudaEventDestroy(p->bfs_done[b]);
+        if (p->copy_done[b]) cudaEventDestroy(p->copy_done[b]);
+    }
+    if (p->copy_stream) cudaStreamDestroy(p->copy_stream);
     if (p->stats_h) cudaFreeHost(p->stats_h);
     if (p->ctr_h) cudaFreeHost(p->ctr_h);
     if (p->l2_window) cudaCtxResetPersistingL2Cache();
@@ -522,6 +532,57 @@ tq_status bfs_plan_wait(bfs_plan *p, bfs_stats *stats)
     if (!p) return TQ_ERR_INVALID;
     DeviceGuard g(p->device);
     return plan_finish(p, stats);
+}
+
+tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
+                             int32_t *level_out, int32_t *parent_out, int64_t out_stride,
+                             bfs_stats *stats)
+{
+    if (!p || !roots || n_roots < 0 || out_stride < 0) return TQ_ERR_INVALID;
+    for (int32_t i = 0; i < n_roots; ++i)
+        if (roots[i] < 0 || roots[i] >= p->n) return TQ_ERR_INVALID;
+    DeviceGuard g(p->device);
+    const bool host_l = level_out && !is_device_ptr(level_out, nullptr);
+    const bool host_p = parent_out && !is_device_ptr(parent_out, nullptr);
+    const size_t vb = (size_t)p->n * sizeof(int32_t);
+    if (host_l || host_p) {
+        // two device output pairs + a copy stream, allocated on first use
+        if (!p->dbuf[0]) {
+            for (int b = 0; b < 2; ++b) CK(cudaMalloc(&p->dbuf[b], 2 * vb));
+            CK(cudaStreamCreateWithFlags(&p->copy_stream, cudaStreamNonBlocking));
+            for (int b = 0; b < 2; ++b) {
+                CK(cudaEventCreateWithFlags(&p->bfs_done[b], cudaEventDisableTiming));
+                CK(cudaEventCreateWithFlags(&p->copy_done[b], cudaEventDisableTiming));
+                CK(cudaEventRecord(p->copy_done[b], p->copy_stream));
+            }
+        }
+    }
+    tq_status st = TQ_OK;
+    for (int32_t i = 0; i < n_roots && st == TQ_OK; ++i) {
+        int32_t *lv = level_out ? level_out + (size_t)i * out_stride : nullptr;
+        int32_t *pa = parent_out ? parent_out + (size_t)i * out_stride : nullptr;
+        if (!host_l && !host_p) {
+            st = plan_launch(p, roots[i], lv, pa);
+            if (st == TQ_OK) st = plan_finish(p, stats ? stats + i : nullptr);
+            continue;
+        }
+        const int b = i & 1;
+        int32_t *dl = lv ? (host_l ? p->dbuf[b] : lv) : nullptr;
+        int32_t *dp = pa ? (host_p ? p->dbuf[b] + p->n : pa) : nullptr;
+        // the buffer pair is free once the copy of root i-2 has drained
+        CK(cudaStreamWaitEvent(p->stream, p->copy_done[b], 0));
+        st = plan_launch(p, roots[i], dl, dp);
+        if (st != TQ_OK) break;
+        CK(cudaEventRecord(p->bfs_done[b], p->stream));
+        CK(cudaStreamWaitEvent(p->copy_stream, p->bfs_done[b], 0));
+        if (host_l) CK(cudaMemcpyAsync(lv, dl, vb, cudaMemcpyDeviceToHost, p->copy_stream));
+        if (host_p) CK(cudaMemcpyAsync(pa, dp, vb, cudaMemcpyDeviceToHost, p->copy_stream));
+        CK(cudaEventRecord(p->copy_done[b], p->copy_stream));
+        // wait for this BFS (the previous root's copy keeps running)
+        st = plan_finish(p, stats ? stats + i : nullptr);
+    }
+    if (p->copy_stream) CK(cudaStreamSynchronize(p->copy_stream));
+    return st;
 }
 
 tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,

@@ -197,6 +197,36 @@ def test_concurrent_plans_on_two_streams(tq):
         p_.close()
 
 
+@pytest.mark.parametrize("where", ["pinned", "pageable", "device"])
+def test_run_batch_overlapped_outputs(tq, where):
+    """bfs_plan_run_batch: one output row per root; host rows are filled by
+    D2H copies overlapped with the next root's BFS."""
+    import torch
+    g = kronecker_csr(12, 16, 9)
+    rp, col = to_dev(g)
+    roots = [int(r) for r in sample_roots(g.row_ptr, 5, 10)]
+    n = g.n_vertices
+    if where == "device":
+        lv = torch.empty(len(roots) * n, dtype=torch.int32, device="cuda")
+        pa = torch.empty_like(lv)
+    elif where == "pinned":
+        lv = torch.empty(len(roots) * n, dtype=torch.int32, pin_memory=True).numpy()
+        pa = torch.empty(len(roots) * n, dtype=torch.int32, pin_memory=True).numpy()
+    else:
+        lv = np.empty(len(roots) * n, dtype=np.int32)
+        pa = np.empty_like(lv)
+    with tq.BfsPlan(rp, col) as plan:
+        stats = plan.run_batch(roots, lv, pa)
+        lvh = lv.cpu().numpy() if where == "device" else lv
+        pah = pa.cpu().numpy() if where == "device" else pa
+        for i, r in enumerate(roots):
+            check_against_oracle(g, r, lvh[i * n:(i + 1) * n], pah[i * n:(i + 1) * n], stats[i])
+        # stride 0: one reused buffer, last root's result remains
+        one = np.empty(n, dtype=np.int32)
+        plan.run_batch(roots, one, None, stride=0)
+        assert np.array_equal(one, oracle.bfs(g.row_ptr, g.col, roots[-1], parents=False)[0])
+
+
 def test_grow_on_full_retries_with_larger_queue(tq):
     g = kronecker_csr(12, 16, 1)
     rp, col = to_dev(g)
