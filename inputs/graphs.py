@@ -190,6 +190,18 @@ def tree4_csr(n: int) -> CSR:
     return edges_to_csr(s, d, n, f"tree4_{n}")
 
 
+def edge_weights(row_ptr, col, seed: int, wmax: int = 255) -> np.ndarray:
+    """Seeded integer edge weights in [1, wmax], one per CSR entry, symmetric
+    (w(u,v) = w(v,u)): h(seed, min(u,v) * 2^32 + max(u,v)) mod wmax + 1."""
+    row_ptr = np.asarray(row_ptr)
+    col = np.asarray(col, dtype=np.int64)
+    rows = np.repeat(np.arange(row_ptr.size - 1, dtype=np.int64), np.diff(row_ptr))
+    lo = np.minimum(rows, col).astype(np.uint64)
+    hi = np.maximum(rows, col).astype(np.uint64)
+    h = hash2(seed ^ 0x77E16475, (lo << np.uint64(32)) | hi)
+    return (h % np.uint64(wmax) + np.uint64(1)).astype(np.int32)
+
+
 def sample_roots(row_ptr: np.ndarray, n_roots: int, seed: int) -> np.ndarray:
     """Graph500-style roots: seeded uniform draws among vertices of degree >= 1.
 

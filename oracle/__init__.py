@@ -59,6 +59,8 @@ def lib() -> ctypes.CDLL:
         L.oracle_traversed_edges.restype = i64
         L.oracle_validate_tree.argtypes = [i64, vp, vp, i32, vp, vp, ctypes.POINTER(i64)]
         L.oracle_validate_tree.restype = ctypes.c_int
+        L.oracle_sssp.argtypes = [i64, vp, vp, vp, i32, vp, vp]
+        L.oracle_sssp.restype = i64
         L.oq_create.argtypes = [u64, u64]
         L.oq_create.restype = vp
         L.oq_destroy.argtypes = [vp]
@@ -137,6 +139,25 @@ def validate_tree(row_ptr, col, root: int, level, parent):
     bad = ctypes.c_int64()
     rule = lib().oracle_validate_tree(rp.size - 1, rpp, cp, int(root), lvp, pap, ctypes.byref(bad))
     return int(rule), int(bad.value)
+
+
+UNREACHED_DIST = 0xFFFFFFFF
+
+
+def sssp(row_ptr, col, weights, src: int):
+    """Dijkstra (oracle.c 4b): returns (dist uint32[V], parent int32[V], reached)."""
+    rp, rpp = _arr(row_ptr, np.int64)
+    c, cp = _arr(col, np.int32)
+    w, wp = _arr(weights, np.int32)
+    if w.size != c.size or (w.size and w.min() < 1):
+        raise ValueError("one weight >= 1 per CSR entry")
+    n = rp.size - 1
+    dist = np.empty(n, dtype=np.uint32)
+    parent = np.empty(n, dtype=np.int32)
+    reached = lib().oracle_sssp(n, rpp, cp, wp, int(src), dist.ctypes.data, parent.ctypes.data)
+    if reached < 0:
+        raise ValueError("oracle_sssp: bad arguments")
+    return dist, parent, int(reached)
 
 
 class QueueModel:

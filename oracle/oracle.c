@@ -179,6 +179,94 @@ int oracle_validate_tree(int64_t n, const int64_t *row_ptr, const int32_t *col, 
 }
 
 /* ------------------------------------------------------------------ */
+/* 4b. Single-source shortest paths (NEXT row 4: the queue reused as a */
+/*     generic scheduler, "it can be used for other purposes with */
+/*     little change").  Textbook Dijkstra with a binary heap (Cormen   */
+/*     et al., the paper's ref. [4], ch. 24) over positive integer      */
+/*     weights w[e] >= 1 of each CSR entry; dist[v] = 0xFFFFFFFF if     */
+/*     unreachable; paths must sum below 2^32 - 1.  parent[v] = the     */
+/*     smallest-id u with dist[u] + w(u->v) == dist[v], parent[src] =   */
+/*     src, -1 unreached (the same tie rule as the BFS min-id parent).  */
+/* ------------------------------------------------------------------ */
+typedef struct { uint64_t key; int32_t v; } oheap_item;
+
+static void oheap_push(oheap_item *h, int64_t *n, uint64_t key, int32_t v)
+{
+    int64_t i = (*n)++;
+    h[i].key = key;
+    h[i].v = v;
+    while (i > 0) {
+        int64_t p = (i - 1) / 2;
+        if (h[p].key <= h[i].key) break;
+        oheap_item t = h[p]; h[p] = h[i]; h[i] = t;
+        i = p;
+    }
+}
+
+static oheap_item oheap_pop(oheap_item *h, int64_t *n)
+{
+    oheap_item top = h[0];
+    h[0] = h[--(*n)];
+    int64_t i = 0;
+    for (;;) {
+        int64_t l = 2 * i + 1, r = l + 1, m = i;
+        if (l < *n && h[l].key < h[m].key) m = l;
+        if (r < *n && h[r].key < h[m].key) m = r;
+        if (m == i) break;
+        oheap_item t = h[m]; h[m] = h[i]; h[i] = t;
+        i = m;
+    }
+    return top;
+}
+
+int64_t oracle_sssp(int64_t n, const int64_t *row_ptr, const int32_t *col, const int32_t *w,
+                    int32_t src, uint32_t *dist, int32_t *parent)
+{
+    if (n <= 0 || src < 0 || src >= n) return -1;
+    const int64_t nnz = row_ptr[n];
+    oheap_item *heap = (oheap_item *)malloc((size_t)(nnz + 1) * sizeof(oheap_item));
+    uint8_t *settled = (uint8_t *)calloc((size_t)n, 1);
+    if (!heap || !settled) { free(heap); free(settled); return -1; }
+    for (int64_t v = 0; v < n; ++v) dist[v] = 0xFFFFFFFFu;
+    int64_t hn = 0, reached = 0;
+    dist[src] = 0;
+    oheap_push(heap, &hn, 0, src);
+    while (hn > 0) {
+        oheap_item it = oheap_pop(heap, &hn);
+        int32_t v = it.v;
+        if (settled[v]) continue;
+        settled[v] = 1;
+        ++reached;
+        for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) {
+            int32_t u = col[e];
+            uint64_t nd = (uint64_t)dist[v] + (uint64_t)(uint32_t)w[e];
+            if (nd < 0xFFFFFFFFull && nd < dist[u]) {
+                dist[u] = (uint32_t)nd;
+                oheap_push(heap, &hn, nd, u);
+            }
+        }
+    }
+    free(heap);
+    free(settled);
+    if (parent) {
+        for (int64_t v = 0; v < n; ++v) parent[v] = -1;
+        parent[src] = src;
+        /* min-id predecessor: scan every edge u->v once */
+        for (int64_t u = 0; u < n; ++u) {
+            if (dist[u] == 0xFFFFFFFFu) continue;
+            for (int64_t e = row_ptr[u]; e < row_ptr[u + 1]; ++e) {
+                int32_t v = col[e];
+                if (v == src) continue;
+                if ((uint64_t)dist[u] + (uint32_t)w[e] == dist[v] &&
+                    (parent[v] < 0 || u < parent[v]))
+                    parent[v] = (int32_t)u;
+            }
+        }
+    }
+    return reached;
+}
+
+/* ------------------------------------------------------------------ */
 /* 5. Sequential ticket model of the RF/AN queue.   */
 /*                                                                     */
 /* State: Front, Rear, capacity C (bounded array) */
