@@ -227,6 +227,25 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
 tq_status bfs_plan_destroy(bfs_plan *p);
 
 /* ------------------------------------------------------------------------ */
+/* The queue as a generic scheduler (NEXT row 4; "it can be used for    */
+/* other purposes with little change"): label-correcting single-source      */
+/* shortest paths on the same persistent kernel, queues and termination.    */
+/* ------------------------------------------------------------------------ */
+
+/* weights: int32[nnz], one per CSR entry, each >= 1 (host or device, like the
+ * CSR; paths must sum below 2^32 - 1).  dist_out[v] = shortest distance
+ * (0xFFFFFFFF unreached); parent_out[v] = the smallest-id u with
+ * dist[u] + w(u->v) == dist[v] (parent_out[src] = src, -1 unreached).  RF_AN
+ * only (opts->variant must be 0); parent_rule is always min-id.  The plan
+ * is destroyed with bfs_plan_destroy. */
+tq_status sssp_plan_create(const tq_csr *g, const int32_t *weights, const bfs_opts *opts,
+                           bfs_plan **out);
+tq_status sssp_plan_run(bfs_plan *p, int32_t src, uint32_t *dist_out, int32_t *parent_out,
+                        bfs_stats *stats);
+tq_status sssp_run_ex(const tq_csr *g, const int32_t *weights, int32_t src, uint32_t *dist_out,
+                      int32_t *parent_out, const bfs_opts *opts, bfs_stats *stats);
+
+/* ------------------------------------------------------------------------ */
 /* Queue micro-benchmark (BASELINE.json configs[1]; Fig 4 / Fig 5 analogue)  */
 /* ------------------------------------------------------------------------ */
 

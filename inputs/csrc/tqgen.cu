@@ -119,6 +119,21 @@ __global__ void keys_to_csr_kernel(const uint64_t *keys, int64_t n_keys, int64_t
     }
 }
 
+// twin of inputs/graphs.py:edge_weights -- one thread per row
+__global__ void edge_weights_kernel(const int64_t *row_ptr, const int32_t *col, int64_t nv,
+                                    uint64_t s_mixed, uint32_t wmax, int32_t *w)
+{
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < nv; v += stride) {
+        for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) {
+            const uint64_t u = (uint64_t)col[e];
+            const uint64_t lo = u < (uint64_t)v ? u : (uint64_t)v, hi = u < (uint64_t)v ? (uint64_t)v : u;
+            const uint64_t h = mix64(s_mixed + ((lo << 32) | hi) * kGolden);
+            w[e] = (int32_t)(h % wmax + 1);
+        }
+    }
+}
+
 int grid_for(int64_t n)
 {
     int dev = 0, sms = 148;
@@ -165,6 +180,16 @@ int tqgen_grid_keys(int64_t rows, int64_t cols, uint64_t *keys, void *stream)
 {
     if (rows < 1 || cols < 1 || !keys) return -1;
     grid_keys_kernel<<<grid_for(rows * cols), 256, 0, (cudaStream_t)stream>>>(rows, cols, keys);
+    return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+// weights: device int32[nnz]; same values as inputs/graphs.py:edge_weights
+int tqgen_edge_weights(const int64_t *row_ptr, const int32_t *col, int64_t nv, uint64_t seed,
+                       uint32_t wmax, int32_t *w, void *stream)
+{
+    if (!row_ptr || nv < 1 || wmax < 1 || !w) return -1;
+    edge_weights_kernel<<<grid_for(nv), 256, 0, (cudaStream_t)stream>>>(
+        row_ptr, col, nv, mix64(seed ^ 0x77E16475ull), wmax, w);
     return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -38,8 +38,9 @@ def lib():
         L.tqgen_tree4_keys.argtypes = [i64, vp, vp]
         L.tqgen_sort_unique.argtypes = [vp, vp, i64, ctypes.POINTER(i64), vp]
         L.tqgen_keys_to_csr.argtypes = [vp, i64, i64, vp, vp, vp]
+        L.tqgen_edge_weights.argtypes = [vp, vp, i64, ctypes.c_uint64, ctypes.c_uint32, vp, vp]
         for f in ("tqgen_kron_keys", "tqgen_grid_keys", "tqgen_tree4_keys", "tqgen_sort_unique",
-                  "tqgen_keys_to_csr"):
+                  "tqgen_keys_to_csr", "tqgen_edge_weights"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -80,6 +81,17 @@ def grid_csr_cuda(rows: int, cols: int | None = None, device="cuda:0"):
     if lib().tqgen_grid_keys(rows, cols, keys.data_ptr(), s):
         raise RuntimeError("tqgen_grid_keys failed")
     return _finish(keys, rows * cols, device)
+
+
+def edge_weights_cuda(row_ptr, col, seed: int, wmax: int = 255):
+    """Twin of inputs.graphs.edge_weights on device tensors."""
+    import torch
+    w = torch.empty(col.numel(), dtype=torch.int32, device=col.device)
+    s = torch.cuda.current_stream(col.device).cuda_stream
+    if lib().tqgen_edge_weights(row_ptr.data_ptr(), col.data_ptr(), row_ptr.numel() - 1,
+                                seed & 0xFFFFFFFFFFFFFFFF, wmax, w.data_ptr(), s):
+        raise RuntimeError("tqgen_edge_weights failed")
+    return w
 
 
 def tree4_csr_cuda(n: int, device="cuda:0"):

@@ -81,6 +81,11 @@ EXPORTS = {
     "bfs_plan_launch": (ctypes.c_int, [c_vp, c_i32, c_vp, c_vp]),
     "bfs_plan_wait": (ctypes.c_int, [c_vp, ctypes.POINTER(bfs_stats)]),
     "bfs_plan_run_batch": (ctypes.c_int, [c_vp, c_vp, c_i32, c_vp, c_vp, c_i64, c_vp]),
+    "sssp_plan_create": (ctypes.c_int, [ctypes.POINTER(tq_csr), c_vp, ctypes.POINTER(bfs_opts),
+                                        ctypes.POINTER(c_vp)]),
+    "sssp_plan_run": (ctypes.c_int, [c_vp, c_i32, c_vp, c_vp, ctypes.POINTER(bfs_stats)]),
+    "sssp_run_ex": (ctypes.c_int, [ctypes.POINTER(tq_csr), c_vp, c_i32, c_vp, c_vp, ctypes.POINTER(bfs_opts),
+                                   ctypes.POINTER(bfs_stats)]),
     "tq_bench": (ctypes.c_int, [ctypes.POINTER(tq_bench_cfg), ctypes.POINTER(tq_bench_result)]),
     "tq_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "tq_persistent_threads": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int,

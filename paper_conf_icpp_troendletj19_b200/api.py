@@ -205,6 +205,54 @@ class BfsPlan:
         self.close()
 
 
+class SsspPlan(BfsPlan):
+    """`sssp_plan_create` / `sssp_plan_run`: label-correcting shortest paths on
+    the same queue and persistent kernel (include/tq.h, NEXT row 4). `weights`
+    is int32[nnz] (>= 1), host or device like the CSR."""
+
+    def __init__(self, row_ptr, col, weights, *, capacity: int = 0, threads: int = 0, chunk: int = 0,
+                 stream=None, timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0,
+                 hub_queue: bool = True):
+        self._w = weights
+        super().__init__(row_ptr, col, variant="rf_an", capacity=capacity, threads=threads, chunk=chunk,
+                         stream=stream, timeout_s=timeout_s, backoff_ns=backoff_ns, device=device,
+                         parents="min_id", hub_queue=hub_queue)
+
+    def _create(self):
+        h = ctypes.c_void_p()
+        check(lib().sssp_plan_create(ctypes.byref(self._g), _ptr(self._w), ctypes.byref(self._opts),
+                                     ctypes.byref(h)), "sssp_plan_create")
+        self._h = h
+
+    def run(self, src: int, dist=None, parent=None, grow_on_full: bool = False) -> dict:
+        """dist: uint32/int32 buffer (0xFFFFFFFF = unreached)."""
+        while True:
+            st = _lib.bfs_stats()
+            status = lib().sssp_plan_run(self._h, int(src), _ptr(dist), _ptr(parent), ctypes.byref(st))
+            if status == _lib.TQ_ERR_QUEUE_FULL and grow_on_full:
+                cap = self._opts.capacity or 2 * max(self.n_vertices, 1 << 15)
+                self._opts.capacity = 2 * max(cap, 1 << 16)
+                self.close()
+                self._create()
+                self.regrows += 1
+                continue
+            check(status, "sssp_plan_run")
+            return _stats_dict(st)
+
+
+def sssp(row_ptr, col, weights, src: int, dist=None, parent=None, **opts):
+    """One-shot shortest paths: returns (dist, parent, stats); dist as int32
+    holding uint32 bits (0xFFFFFFFF = unreached)."""
+    n = int(row_ptr.shape[0]) - 1
+    if dist is None:
+        dist = _empty_like_graph(row_ptr, n)
+    if parent is None:
+        parent = _empty_like_graph(row_ptr, n)
+    with SsspPlan(row_ptr, col, weights, **opts) as p:
+        st = p.run(src, dist, parent)
+    return dist, parent, st
+
+
 def run_concurrent(plans, roots, levels=None, parents=None):
     """Run `roots` over several plans (each on its own stream) keeping one BFS
     in flight per plan; returns the per-root statistics in root order."""

@@ -107,6 +107,10 @@ struct bfs_plan {
     int32_t *hub_base = nullptr;
     uint8_t *lvl8 = nullptr;
     uint8_t *x8 = nullptr;
+    unsigned *xd = nullptr;                   // SSSP: expanded-distance marker
+    int32_t *wgt = nullptr;                   // SSSP: edge weights (device)
+    bool owns_wgt = false;
+    int task = 0;                             // kTaskBFS / kTaskSSSP
     int2 *chunk_tab = nullptr;
     int64_t n_chunks = 0;
     tq_queue *q = nullptr;
@@ -261,6 +265,8 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     cudaFree(p->hub_base);
     cudaFree(p->lvl8);
     cudaFree(p->x8);
+    cudaFree(p->xd);
+    if (p->owns_wgt) cudaFree(p->wgt);
     cudaFree(p->chunk_tab);
     cudaFree(p->stats);
     cudaFree(p->out_scratch);
@@ -281,7 +287,8 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     return TQ_OK;
 }
 
-tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **out)
+static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int task,
+                                  const bfs_opts *opts, bfs_plan **out)
 {
     if (!gph || !out) return TQ_ERR_INVALID;
     *out = nullptr;
@@ -292,6 +299,8 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (n < 1 || n >= (1ll << 31) || nnz < 0 || !gph->row_ptr || (nnz > 0 && !gph->col))
         return TQ_ERR_INVALID;
     if (o.variant < TQ_VARIANT_RF_AN || o.variant > TQ_VARIANT_AN) return TQ_ERR_UNSUPPORTED;
+    if (task == kTaskSSSP && o.variant != TQ_VARIANT_RF_AN) return TQ_ERR_UNSUPPORTED;
+    if (task == kTaskSSSP && nnz > 0 && !weights) return TQ_ERR_INVALID;
     int chunk = o.chunk ? o.chunk : 512;
     if (chunk < 32 || chunk > 65536 || (chunk & (chunk - 1))) return TQ_ERR_INVALID;
     const int block = o.block ? o.block : 256;
@@ -316,7 +325,8 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
         delete p;
         return TQ_ERR_INVALID;
     }
-    p->parent_rule = o.parent_rule;
+    p->parent_rule = task == kTaskSSSP ? TQ_PARENT_MIN_ID : o.parent_rule;
+    p->task = task;
     p->n = n;
     p->nnz = nnz;
 
@@ -340,10 +350,26 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
                                 cudaMemcpyHostToDevice, p->stream);
         if (e != cudaSuccess) return fail(from_cuda(e));
     }
+    if (task == kTaskSSSP && nnz > 0) {
+        if (is_device_ptr(weights, nullptr)) {
+            p->wgt = const_cast<int32_t *>(weights);
+        } else {
+            p->owns_wgt = true;
+            e = cudaMalloc(&p->wgt, (size_t)nnz * sizeof(int32_t));
+            if (e == cudaSuccess)
+                e = cudaMemcpyAsync(p->wgt, weights, (size_t)nnz * sizeof(int32_t), cudaMemcpyHostToDevice,
+                                    p->stream);
+            if (e != cudaSuccess) return fail(from_cuda(e));
+        }
+    }
     e = cudaMalloc(&p->W, (size_t)n * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMalloc(&p->hub_base, (size_t)n * sizeof(int32_t));
-    if (e == cudaSuccess) e = cudaMalloc(&p->lvl8, (size_t)n);
-    if (e == cudaSuccess) e = cudaMalloc(&p->x8, (size_t)n);
+    if (task == kTaskBFS) {
+        if (e == cudaSuccess) e = cudaMalloc(&p->lvl8, (size_t)n);
+        if (e == cudaSuccess) e = cudaMalloc(&p->x8, (size_t)n);
+    } else {
+        if (e == cudaSuccess) e = cudaMalloc(&p->xd, (size_t)n * sizeof(unsigned));
+    }
     if (e == cudaSuccess) e = cudaMalloc(&p->stats, kStatCount * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMallocHost(&p->ctr_h, 8 * sizeof(unsigned long long));
@@ -354,7 +380,9 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (e != cudaSuccess) return fail(from_cuda(e));
     if (n + p->n_chunks >= (1ll << 31)) return fail(TQ_ERR_UNSUPPORTED);
 
-    uint64_t cap = o.capacity ? o.capacity : next_pow2((uint64_t)(2 * n));
+    // weighted label correcting re-enqueues far more than BFS: 8V for SSSP
+    uint64_t cap = o.capacity ? o.capacity : next_pow2((uint64_t)((task == kTaskSSSP ? 8 : 2) * n));
+    if (cap > (1ull << 31)) cap = 1ull << 31;
     if (!o.capacity && cap < (1ull << 16)) cap = 1ull << 16;
     tq_status st = tq_create(cap, gdev, &p->q);
     if (st != TQ_OK) return fail(st);
@@ -380,7 +408,7 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
         p->blocks = full;
     }
     if (p->blocks < 1) p->blocks = 1;
-    {
+    if (task == kTaskBFS) {
         // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the byte
         // mirror is probed once per edge; a persisting window keeps it
         // resident against the col stream.  The device-wide carve-out is
@@ -405,6 +433,17 @@ tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **ou
     if (e != cudaSuccess) return fail(from_cuda(e));
     *out = p;
     return TQ_OK;
+}
+
+tq_status bfs_plan_create(const tq_csr *gph, const bfs_opts *opts, bfs_plan **out)
+{
+    return plan_create_impl(gph, nullptr, kTaskBFS, opts, out);
+}
+
+tq_status sssp_plan_create(const tq_csr *gph, const int32_t *weights, const bfs_opts *opts,
+                           bfs_plan **out)
+{
+    return plan_create_impl(gph, weights, kTaskSSSP, opts, out);
 }
 
 // First half of a run: enqueue init + persistent kernel + unpack and the
@@ -438,6 +477,9 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.hub_base = p->hub_base;
     bp.lvl8 = p->lvl8;
     bp.x8 = p->x8;
+    bp.xd = p->xd;
+    bp.wgt = p->wgt;
+    bp.task = p->task;
     bp.parent_rule = p->parent_rule;
     bp.stats = p->stats;
     bp.n_vertices = p->n;
@@ -625,6 +667,26 @@ tq_status bfs_run_ex(const tq_csr *g, int32_t root, int32_t *level_out, int32_t 
 tq_status bfs_run(const tq_csr *g, int32_t root, int32_t *level_out, int32_t *parent_out)
 {
     return bfs_run_ex(g, root, level_out, parent_out, nullptr, nullptr);
+}
+
+tq_status sssp_plan_run(bfs_plan *p, int32_t src, uint32_t *dist_out, int32_t *parent_out,
+                        bfs_stats *stats)
+{
+    if (!p || p->task != kTaskSSSP) return TQ_ERR_INVALID;
+    // the unpack writes dist's 32 bits (0xFFFFFFFF = unreached) into dist_out
+    return bfs_plan_run(p, src, reinterpret_cast<int32_t *>(dist_out), parent_out, stats);
+}
+
+tq_status sssp_run_ex(const tq_csr *g, const int32_t *weights, int32_t src, uint32_t *dist_out,
+                      int32_t *parent_out, const bfs_opts *opts, bfs_stats *stats)
+{
+    if (!g || src < 0 || src >= g->n_vertices) return TQ_ERR_INVALID;
+    bfs_plan *p = nullptr;
+    tq_status st = sssp_plan_create(g, weights, opts, &p);
+    if (st != TQ_OK) return st;
+    st = sssp_plan_run(p, src, dist_out, parent_out, stats);
+    bfs_plan_destroy(p);
+    return st;
 }
 
 // ------------------------------------------------------------------------

@@ -364,7 +364,7 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
 // ---------------------------------------------------------------------------
 // The persistent kernel
 // ---------------------------------------------------------------------------
-template <int VARIANT, int KU = kU, int MINB = kMinBlocks>
+template <int VARIANT, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks>
 __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsParams p)
 {
     __shared__ uint32_t stage_all[kWarps][kStageCap];
@@ -561,6 +561,20 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
             // current cost of the node (Listing 2 line 21), read fresh
             const unsigned L = (unsigned)(tq_ld_relaxed(p.W + v) >> 32);
+            if constexpr (TASK == kTaskSSSP) {
+                // the edge weight is added per edge in the expansion
+                offer = ((unsigned long long)L << 32) | (unsigned)v;
+                if (!(item & CHUNK_FLAG)) {  // expanded-distance marker (R7 for SSSP)
+                    const unsigned xprev = (unsigned)ld_relaxed_i32((const int32_t *)p.xd + v);
+                    if (xprev <= L) {
+                        skipped = true;
+                        hi = lo;
+                        nch = 0;
+                    } else {
+                        st_relaxed_i32((int32_t *)p.xd + v, (int)L);
+                    }
+                }
+            } else {
             offer = ((unsigned long long)(L + 1) << 32) | (unsigned)v;
             if (!(item & CHUNK_FLAG)) {
                 // expanded-level marker (R7): a vertex already
@@ -576,6 +590,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 } else {
                     st_u8(p.x8 + v, L < kLvlSat ? L : kLvlSat);
                 }
+            }
             }
         }
 
@@ -616,7 +631,24 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 const long long eb = (long long)tq_shfl64((unsigned long long)ebase, o);
                 off[j] = tq_shfl64(offer, o);
                 u[j] = val[j] ? ld_nc_i32(p.col + eb + gg, pol_stream) : 0;
+                if constexpr (TASK == kTaskSSSP) {
+                    const unsigned wt = val[j] ? (unsigned)ld_nc_i32(p.wgt + eb + gg, pol_stream) : 0u;
+                    const unsigned long long d = (off[j] >> 32) + wt;  // dist(v) + w(v -> u)
+                    val[j] = val[j] && d < 0xffffffffull;
+                    off[j] = (d << 32) | (off[j] & 0xffffffffull);
+                }
             }
+            bool cand[KU];
+            if constexpr (TASK == kTaskSSSP) {
+                // prefilter: the packed word itself (dist, parent) -- stale
+                // values are never below the true word, so skipping offers
+                // that do not beat it drops no improvement
+                unsigned long long w[KU];
+#pragma unroll
+                for (int j = 0; j < KU; ++j) w[j] = val[j] ? ld_cg_u64(p.W + u[j]) : 0ull;
+#pragma unroll
+                for (int j = 0; j < KU; ++j) cand[j] = val[j] && off[j] < w[j];
+            } else {
             // prefilter 1: the byte level mirror (L2-resident; stale values
             // are never below the true level, R8)
             unsigned m8[KU];
@@ -628,7 +660,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 const bool deep = (unsigned)(off[j] >> 32) >= kLvlSat;
                 m8[j] = (val[j] && !deep) ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : kLvlSat;
             }
-            bool cand[KU], tie[KU];
+            bool tie[KU];
 #pragma unroll
             for (int j = 0; j < KU; ++j) {
                 const unsigned L1 = (unsigned)(off[j] >> 32);
@@ -648,6 +680,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 #pragma unroll
                 for (int j = 0; j < KU; ++j) cand[j] = cand[j] || (tie[j] && off[j] < w[j]);
             }
+            }
             bool nt[KU];
             unsigned n_min = 0, n_reenq = 0;
 #pragma unroll
@@ -659,7 +692,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     const unsigned L1 = (unsigned)(off[j] >> 32);
                     if ((old >> 32) > L1) {  // level strictly lowered: (re)discovered
                         nt[j] = true;
-                        st_u8(p.lvl8 + u[j], L1 < kLvlSat ? L1 : kLvlSat);
+                        if constexpr (TASK == kTaskBFS) st_u8(p.lvl8 + u[j], L1 < kLvlSat ? L1 : kLvlSat);
                         re = (old >> 32) != 0xffffffffull;
                     }
                 }
@@ -748,8 +781,9 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
         p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
-        p.lvl8[i] = (i == root) ? 0 : 255;
-        p.x8[i] = 255;
+        if (p.lvl8) p.lvl8[i] = (i == root) ? 0 : 255;
+        if (p.x8) p.x8[i] = 255;
+        if (p.xd) p.xd[i] = 0xffffffffu;
     }
     if (blockIdx.x == 0) {
         if (threadIdx.x < TQ_STATUS_COPIES) p.q.status[threadIdx.x * TQ_STATUS_STRIDE] = TQ_RUNNING;
@@ -894,7 +928,7 @@ cudaError_t launch_queue_reset(const tq_device_view &q, cudaStream_t s)
     return cudaGetLastError();
 }
 
-template <int V, int KU = kU, int MINB = kMinBlocks>
+template <int V, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks>
 static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStream_t s)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
@@ -916,12 +950,16 @@ static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStrea
         cfg.attrs = attr;
         cfg.numAttrs = 1;
     }
-    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, KU, MINB>, p);
+    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, TASK, KU, MINB>, p);
 }
 
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
                                   cudaStream_t s)
 {
+    if (p.task == kTaskSSSP) {  // the generic-scheduler row runs on the RF/AN queue
+        if (variant != TQ_VARIANT_RF_AN) return cudaErrorInvalidValue;
+        return launch_v<TQ_VARIANT_RF_AN, kTaskSSSP>(p, blocks, block, s);
+    }
     switch (variant) {
     case TQ_VARIANT_RF_AN: return launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
     case TQ_VARIANT_PER_THREAD_AFA: return launch_v<TQ_VARIANT_PER_THREAD_AFA>(p, blocks, block, s);

@@ -30,6 +30,10 @@ __device__ __forceinline__ unsigned long long *per_lane_addr(unsigned long long 
 }
 
 constexpr int kStatCount = 16;
+
+// Task run by the persistent kernel over the queue (the queue is the same).
+constexpr int kTaskBFS = 0;   // top-down BFS levels (the paper's driver)
+constexpr int kTaskSSSP = 1;  // label-correcting shortest paths (NEXT row 4)
 enum StatIndex {
     ST_TASKS = 0,
     ST_CHUNK_TASKS,
@@ -61,6 +65,9 @@ struct BfsParams {
     const int32_t *hub_base;   // vertex -> first chunk id (read for hubs only)
     uint8_t *lvl8;             // byte level mirror (prefilter), 255 = unreached
     uint8_t *x8;               // level at which the vertex was expanded (saturating byte)
+    unsigned *xd;              // SSSP: distance at which the vertex was expanded
+    const int32_t *wgt;        // SSSP: edge weights (one per CSR entry), else null
+    int task;                  // kTaskBFS / kTaskSSSP
     unsigned long long *stats; // kStatCount counters
     int64_t n_vertices;
     int chunk;                 // max edges per token (power of 2)

@@ -22,6 +22,14 @@ def test_kronecker_twin(gen, scale, seed):
     assert np.array_equal(col.cpu().numpy(), a.col)
 
 
+def test_edge_weight_twin(gen):
+    from inputs import edge_weights
+    a = kronecker_csr(12, 16, 2)
+    rp, col = gen.kronecker_csr_cuda(12, 16, 2)
+    w = gen.edge_weights_cuda(rp, col, 7, 255)
+    assert np.array_equal(w.cpu().numpy(), edge_weights(a.row_ptr, a.col, 7, 255))
+
+
 def test_grid_and_tree_twins(gen):
     a = grid_csr(37, 53)
     rp, col = gen.grid_csr_cuda(37, 53)
