@@ -64,6 +64,23 @@ int is_device_ptr(const void *p, int *device)
     return 0;
 }
 
+// Device -> host copy in 8 MiB pieces.  Measured on the B200 boxes
+// (scripts/overlap_probe.cu): while ONE large D2H copy is in flight, a
+// multi-CTA kernel launched after it does not start until the copy ends
+// (a 512 MiB copy delays the next BFS by ~10 ms); split into 8 MiB copies
+// the kernel starts at once and the copy still runs at ~52 GB/s.
+static cudaError_t d2h_chunked(void *dst, const void *src, size_t bytes, cudaStream_t s)
+{
+    const size_t piece = 8ull << 20;
+    for (size_t off = 0; off < bytes; off += piece) {
+        const size_t nb = bytes - off < piece ? bytes - off : piece;
+        cudaError_t e = cudaMemcpyAsync((char *)dst + off, (const char *)src + off, nb,
+                                        cudaMemcpyDeviceToHost, s);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
 uint64_t next_pow2(uint64_t x)
 {
     uint64_t c = 1;
@@ -408,7 +425,8 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         p->blocks = full;
     }
     if (p->blocks < 1) p->blocks = 1;
-    if (task == kTaskBFS) {
+    const char *l2env = getenv("TQ_L2_WINDOW");  // "0": experiments only
+    if (task == kTaskBFS && !(l2env && l2env[0] == '0')) {
         // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the byte
         // mirror is probed once per edge; a persisting window keeps it
         // resident against the col stream.  The device-wide carve-out is
@@ -600,6 +618,22 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
         }
     }
     tq_status st = TQ_OK;
+    // Host outputs: root i's arrays drain (copy stream) while root i+1 runs.
+    // The copy of root i is issued AFTER root i+1's kernels are enqueued:
+    // measured on the B200 boxes, a persistent BFS enqueued while a large
+    // D2H copy is in flight does not start until the copy ends, whereas a
+    // copy enqueued behind the running kernel overlaps it fully.
+    int32_t pend = -1;  // root whose outputs still have to be copied
+    auto issue_copy = [&](int32_t k) -> cudaError_t {
+        const int b = k & 1;
+        int32_t *lv = level_out + (level_out ? (size_t)k * out_stride : 0);
+        int32_t *pa = parent_out + (parent_out ? (size_t)k * out_stride : 0);
+        cudaError_t e = cudaStreamWaitEvent(p->copy_stream, p->bfs_done[b], 0);
+        if (e == cudaSuccess && host_l) e = d2h_chunked(lv, p->dbuf[b], vb, p->copy_stream);
+        if (e == cudaSuccess && host_p) e = d2h_chunked(pa, p->dbuf[b] + p->n, vb, p->copy_stream);
+        if (e == cudaSuccess) e = cudaEventRecord(p->copy_done[b], p->copy_stream);
+        return e;
+    };
     for (int32_t i = 0; i < n_roots && st == TQ_OK; ++i) {
         int32_t *lv = level_out ? level_out + (size_t)i * out_stride : nullptr;
         int32_t *pa = parent_out ? parent_out + (size_t)i * out_stride : nullptr;
@@ -616,13 +650,11 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
         st = plan_launch(p, roots[i], dl, dp);
         if (st != TQ_OK) break;
         CK(cudaEventRecord(p->bfs_done[b], p->stream));
-        CK(cudaStreamWaitEvent(p->copy_stream, p->bfs_done[b], 0));
-        if (host_l) CK(cudaMemcpyAsync(lv, dl, vb, cudaMemcpyDeviceToHost, p->copy_stream));
-        if (host_p) CK(cudaMemcpyAsync(pa, dp, vb, cudaMemcpyDeviceToHost, p->copy_stream));
-        CK(cudaEventRecord(p->copy_done[b], p->copy_stream));
-        // wait for this BFS (the previous root's copy keeps running)
+        if (pend >= 0) CK(issue_copy(pend));
+        pend = i;
         st = plan_finish(p, stats ? stats + i : nullptr);
     }
+    if (pend >= 0 && st == TQ_OK) CK(issue_copy(pend));
     if (p->copy_stream) CK(cudaStreamSynchronize(p->copy_stream));
     return st;
 }
@@ -645,9 +677,9 @@ tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *p
     if (st == TQ_OK) st = plan_finish(p, stats);
     if (st != TQ_OK) return st;
     if (host_l)
-        CK(cudaMemcpyAsync(level_out, dl, (size_t)p->n * sizeof(int32_t), cudaMemcpyDeviceToHost, p->stream));
+        CK(d2h_chunked(level_out, dl, (size_t)p->n * sizeof(int32_t), p->stream));
     if (host_p)
-        CK(cudaMemcpyAsync(parent_out, dp, (size_t)p->n * sizeof(int32_t), cudaMemcpyDeviceToHost, p->stream));
+        CK(d2h_chunked(parent_out, dp, (size_t)p->n * sizeof(int32_t), p->stream));
     CK(cudaStreamSynchronize(p->stream));
     return TQ_OK;
 }
