@@ -23,6 +23,7 @@
 #ifndef TQ_H_
 #define TQ_H_
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -158,6 +159,13 @@ typedef struct {
                            second RF/AN queue that lane 0 of every warp polls
                            first (0 = default on, < 0 = off: chunks share the
                            main queue).  Ignored by the other variants.     */
+    int debug_delay_ns; /* TEST ONLY (schedule perturbation, SURVEY §8(c)
+                           "schedule independence"): the lane holding vertex
+                           v sleeps this long before reading v's level when
+                           mix(v ^ seed) % 8 == 0, and after reading it when
+                           == 1, so tokens are expanded late and with stale
+                           levels.  0 = off (default); at most 1,000,000     */
+    uint32_t debug_delay_seed;
 } bfs_opts;
 
 enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };
@@ -288,6 +296,10 @@ const char *tq_strerror(tq_status s);
 tq_status tq_persistent_threads(int variant, int block, int device, int *threads_out);
 /* Library version string. */
 const char *tq_version(void);
+/* sizeof() of a public struct by name ("tq_csr", "bfs_opts", "bfs_stats",
+ * "tq_device_view", "tq_counters", "tq_bench_cfg", "tq_bench_result"), 0 for
+ * an unknown name: lets bindings check their struct mirrors without a GPU. */
+size_t tq_struct_size(const char *name);
 
 #ifdef __cplusplus
 }

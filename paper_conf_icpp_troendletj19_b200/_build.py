@@ -36,17 +36,20 @@ def up_to_date(lib: str, inputs: list[str]) -> bool:
     return all(os.path.getmtime(d) <= t for d in inputs)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date(LIB, deps()):
-        return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), "-o", tmp, *sources()]
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Build libtq.so (or, for A/B experiments, `out` with extra -D `defines`)."""
+    lib = out or LIB
+    if not force and up_to_date(lib, deps()):
+        return lib
+    tmp = lib + f".tmp{os.getpid()}"
+    cmd = [NVCC, *ARCH, *FLAGS, *(f"-D{d}" for d in defines), "-I", os.path.join(ROOT, "include"), "-o", tmp,
+           *sources()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd))
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":

@@ -39,7 +39,8 @@ class bfs_opts(ctypes.Structure):
     _fields_ = [("capacity", c_u64), ("threads", ctypes.c_int), ("block", ctypes.c_int),
                 ("chunk", ctypes.c_int), ("variant", ctypes.c_int), ("stream", c_vp),
                 ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int),
-                ("parent_rule", ctypes.c_int), ("hub_queue", ctypes.c_int)]
+                ("parent_rule", ctypes.c_int), ("hub_queue", ctypes.c_int),
+                ("debug_delay_ns", ctypes.c_int), ("debug_delay_seed", c_u32)]
 
 
 class bfs_stats(ctypes.Structure):
@@ -92,7 +93,11 @@ EXPORTS = {
     "tq_persistent_threads": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                              ctypes.POINTER(ctypes.c_int)]),
     "tq_version": (ctypes.c_char_p, []),
+    "tq_struct_size": (ctypes.c_size_t, [ctypes.c_char_p]),
 }
+
+STRUCTS = {"tq_csr": tq_csr, "bfs_opts": bfs_opts, "bfs_stats": bfs_stats, "tq_device_view": tq_device_view,
+           "tq_counters": tq_counters, "tq_bench_cfg": tq_bench_cfg, "tq_bench_result": tq_bench_result}
 
 _lib = None
 

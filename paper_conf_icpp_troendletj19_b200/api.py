@@ -74,11 +74,12 @@ def _csr(row_ptr, col) -> _lib.tq_csr:
 
 
 def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None, timeout_s=0.0,
-          backoff_ns=0, device=0, parents="any", hub_queue=True) -> _lib.bfs_opts:
+          backoff_ns=0, device=0, parents="any", hub_queue=True, debug_delay_ns=0,
+          debug_delay_seed=0) -> _lib.bfs_opts:
     return _lib.bfs_opts(int(capacity), int(threads), int(block), int(chunk), _variant(variant),
                          stream, float(timeout_s), int(backoff_ns), int(device),
                          _lib.PARENT_RULES[parents] if isinstance(parents, str) else int(parents),
-                         0 if hub_queue else -1)
+                         0 if hub_queue else -1, int(debug_delay_ns), int(debug_delay_seed) & 0xFFFFFFFF)
 
 
 def _stats_dict(st: _lib.bfs_stats) -> dict:
@@ -95,7 +96,7 @@ def _empty_like_graph(row_ptr, n):
 def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool = True,
         variant="rf_an", capacity: int = 0, threads: int = 0, chunk: int = 0, stream=None,
         timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0, parents="any",
-        hub_queue: bool = True):
+        hub_queue: bool = True, debug_delay_ns: int = 0, debug_delay_seed: int = 0):
     """One-shot `bfs_run_ex`: returns (level, parent, stats).
 
     Graph arrays may be CUDA tensors (used in place) or host numpy arrays
@@ -110,7 +111,7 @@ def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool =
         parent = _empty_like_graph(row_ptr, n)
     o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
               backoff_ns, row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device,
-              parents, hub_queue)
+              parents, hub_queue, debug_delay_ns, debug_delay_seed)
     st = _lib.bfs_stats()
     check(lib().bfs_run_ex(ctypes.byref(g), int(root), _ptr(level), _ptr(parent), ctypes.byref(o),
                            ctypes.byref(st)), "bfs_run_ex")
@@ -126,14 +127,16 @@ class BfsPlan:
 
     def __init__(self, row_ptr, col, *, variant="rf_an", capacity: int = 0, threads: int = 0,
                  chunk: int = 0, stream=None, timeout_s: float = 0.0, backoff_ns: int = 0,
-                 device: int = 0, parents="any", hub_queue: bool = True):
+                 device: int = 0, parents="any", hub_queue: bool = True, debug_delay_ns: int = 0,
+                 debug_delay_seed: int = 0):
         self._keep = (row_ptr, col)  # device arrays must outlive the plan
         self._g = _csr(row_ptr, col)
         self.n_vertices = self._g.n_vertices
         self.nnz = self._g.nnz
         self.device = row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device
         self._opts = o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr),
-                               timeout_s, backoff_ns, self.device, parents, hub_queue)
+                               timeout_s, backoff_ns, self.device, parents, hub_queue, debug_delay_ns,
+                               debug_delay_seed)
         self.regrows = 0
         self._h = None
         self._create()
@@ -212,11 +215,12 @@ class SsspPlan(BfsPlan):
 
     def __init__(self, row_ptr, col, weights, *, capacity: int = 0, threads: int = 0, chunk: int = 0,
                  stream=None, timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0,
-                 hub_queue: bool = True):
+                 hub_queue: bool = True, debug_delay_ns: int = 0, debug_delay_seed: int = 0):
         self._w = weights
         super().__init__(row_ptr, col, variant="rf_an", capacity=capacity, threads=threads, chunk=chunk,
                          stream=stream, timeout_s=timeout_s, backoff_ns=backoff_ns, device=device,
-                         parents="min_id", hub_queue=hub_queue)
+                         parents="min_id", hub_queue=hub_queue, debug_delay_ns=debug_delay_ns,
+                         debug_delay_seed=debug_delay_seed)
 
     def _create(self):
         h = ctypes.c_void_p()

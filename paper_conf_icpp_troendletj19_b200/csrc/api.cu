@@ -147,12 +147,27 @@ struct bfs_plan {
     unsigned long long next_ticket = 0;
     bool dirty = false;
     int32_t *out_scratch = nullptr;           // for host outputs
+    int delay_ns = 0;                         // test only (bfs_opts.debug_delay_ns)
+    uint32_t delay_seed = 0;
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
 };
 
 extern "C" {
 
 const char *tq_version(void) { return TQ_VERSION_STRING; }
+
+size_t tq_struct_size(const char *name)
+{
+    if (!name) return 0;
+    if (!strcmp(name, "tq_csr")) return sizeof(tq_csr);
+    if (!strcmp(name, "bfs_opts")) return sizeof(bfs_opts);
+    if (!strcmp(name, "bfs_stats")) return sizeof(bfs_stats);
+    if (!strcmp(name, "tq_device_view")) return sizeof(tq_device_view);
+    if (!strcmp(name, "tq_counters")) return sizeof(tq_counters);
+    if (!strcmp(name, "tq_bench_cfg")) return sizeof(tq_bench_cfg);
+    if (!strcmp(name, "tq_bench_result")) return sizeof(tq_bench_result);
+    return 0;
+}
 
 const char *tq_strerror(tq_status s)
 {
@@ -343,6 +358,12 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         return TQ_ERR_INVALID;
     }
     p->parent_rule = task == kTaskSSSP ? TQ_PARENT_MIN_ID : o.parent_rule;
+    if (o.debug_delay_ns < 0 || o.debug_delay_ns > 1000000) {
+        delete p;
+        return TQ_ERR_INVALID;
+    }
+    p->delay_ns = o.debug_delay_ns;
+    p->delay_seed = o.debug_delay_seed;
     p->task = task;
     p->n = n;
     p->nnz = nnz;
@@ -506,6 +527,8 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.backoff_ns = p->backoff_ns;
     bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
     bp.l2_window_bytes = p->l2_window;
+    bp.delay_ns = (unsigned)p->delay_ns;
+    bp.delay_seed = p->delay_seed;
 
     CK(cudaEventRecord(p->ev[0], s));
     CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));

@@ -85,6 +85,15 @@ __device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long lon
     asm volatile("ld.global.cg.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
+__device__ __forceinline__ unsigned mix32(unsigned x)
+{
+    x ^= x >> 16;
+    x *= 0x7feb352du;
+    x ^= x >> 15;
+    x *= 0x846ca68bu;
+    x ^= x >> 16;
+    return x;
+}
 __device__ __forceinline__ unsigned ld_relaxed_u8(const uint8_t *p)
 {
     unsigned v;
@@ -559,8 +568,15 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     hi = lo;
                 }
             }
+            // test-only schedule perturbation (bfs_opts.debug_delay_ns)
+            unsigned dly = 8;
+            if (p.delay_ns) {
+                dly = (unsigned)(mix32((unsigned)v ^ p.delay_seed) & 7u);
+                if (dly == 0) __nanosleep(p.delay_ns);
+            }
             // current cost of the node (Listing 2 line 21), read fresh
             const unsigned L = (unsigned)(tq_ld_relaxed(p.W + v) >> 32);
+            if (dly == 1) __nanosleep(p.delay_ns);
             if constexpr (TASK == kTaskSSSP) {
                 // the edge weight is added per edge in the expansion
                 offer = ((unsigned long long)L << 32) | (unsigned)v;

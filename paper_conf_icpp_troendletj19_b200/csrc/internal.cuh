@@ -76,6 +76,8 @@ struct BfsParams {
     int parent_rule;           // TQ_PARENT_ANY / TQ_PARENT_MIN_ID (include/tq.h)
     unsigned long long timeout_ns;
     size_t l2_window_bytes;    // persisting-L2 window over lvl8 (0 = none)
+    unsigned delay_ns;         // test only: schedule perturbation (bfs_opts.debug_delay_ns)
+    unsigned delay_seed;
 };
 
 // bfs.cu

@@ -46,6 +46,16 @@ def test_library_loads_and_reports(libtq):
     assert L.tq_strerror(-4).startswith(b"queue full")
 
 
+def test_struct_mirrors_match_the_header(libtq):
+    """Every ctypes mirror has the C layout's size (include/tq.h)."""
+    import ctypes
+    from paper_conf_icpp_troendletj19_b200 import _lib
+    L = _lib.lib()
+    for name, cls in _lib.STRUCTS.items():
+        assert L.tq_struct_size(name.encode()) == ctypes.sizeof(cls), name
+    assert L.tq_struct_size(b"no_such_struct") == 0
+
+
 def test_library_is_sm_100a_code(libtq):
     out = subprocess.check_output(["cuobjdump", "--list-elf", libtq], text=True)
     assert "sm_100a" in out

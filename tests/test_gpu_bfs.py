@@ -136,6 +136,41 @@ def test_label_correcting_motif(tq):
         check_against_oracle(g, 0, level, parent, st)
 
 
+@pytest.mark.parametrize("parents", ["any", "min_id"])
+@pytest.mark.parametrize("variant", ["rf_an", "an"])
+def test_schedule_independence_under_delay_injection(tq, variant, parents):
+    """SURVEY §8(c) "schedule independence": with the test-only delay
+    injection (bfs_opts.debug_delay_ns) 1/8 of the vertices are expanded late
+    and another 1/8 with a level read long before their offers land, for
+    several seeds: levels stay identical to the oracle, parents identical
+    under min-id and valid under 'any' (label correcting, R4)."""
+    n = 6 + 200
+    src = [0, 0, 1, 3, 2] + [1] + list(range(6, n - 1))
+    dst = [1, 2, 3, 4, 4] + [6] + list(range(7, n))
+    graphs = [edges_to_csr(np.array(src), np.array(dst), n), kronecker_csr(11, 16, 7), grid_csr(48, 37),
+              tree4_csr(3000)]
+    for g in graphs:
+        rp, col = to_dev(g)
+        root = int(sample_roots(g.row_ptr, 1, 3)[0]) if g.n_vertices > 5000 else 0
+        for seed in range(4):
+            level, parent, st = tq.bfs(rp, col, root, variant=variant, parents=parents, timeout_s=30,
+                                       chunk=64, debug_delay_ns=20000, debug_delay_seed=seed)
+            check_against_oracle(g, root, level, parent, st, min_id=parents == "min_id")
+
+
+def test_delay_injection_perturbs_the_schedule(tq):
+    """The injection really changes the execution: on the motif graph with a
+    slow path the delayed runs re-enqueue (level corrections) or take longer."""
+    g = kronecker_csr(12, 16, 3)
+    rp, col = to_dev(g)
+    root = int(sample_roots(g.row_ptr, 1, 4)[0])
+    _, _, st0 = tq.bfs(rp, col, root)
+    _, _, st1 = tq.bfs(rp, col, root, debug_delay_ns=50000, debug_delay_seed=1)
+    assert st1["ms_kernel"] > st0["ms_kernel"]
+    with pytest.raises(tq.TQError):
+        tq.bfs(rp, col, root, debug_delay_ns=2_000_000)  # out of range -> TQ_ERR_INVALID
+
+
 @pytest.mark.parametrize("chunk", [32, 64, 1024])
 def test_hub_chunking(tq, chunk):
     """Vertices with more than `chunk` edges are split into chunk tokens."""

@@ -76,3 +76,16 @@ def test_sssp_rejects_other_variants(tq):
         h = ctypes.c_void_p()
         _lib.check(_lib.lib().sssp_plan_create(ctypes.byref(api._csr(g.row_ptr, g.col)), w.ctypes.data,
                                                ctypes.byref(o), ctypes.byref(h)), "sssp_plan_create")
+
+
+def test_sssp_schedule_independence_under_delay_injection(tq):
+    """Delay injection (bfs_opts.debug_delay_ns): distances and
+    min-id parents stay identical to Dijkstra under perturbed schedules."""
+    for g in (kronecker_csr(11, 16, 4), grid_csr(40, 33)):
+        w = edge_weights(g.row_ptr, g.col, 5, 100)
+        rp, col, wd = dev(g.row_ptr), dev(g.col), dev(w)
+        src = int(np.argmax(g.degrees()))
+        for seed in range(3):
+            dist, parent, _ = tq.sssp(rp, col, wd, src, chunk=64, timeout_s=30, debug_delay_ns=20000,
+                                      debug_delay_seed=seed)
+            check(g, w, src, dist, parent)
