@@ -441,7 +441,7 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     if (e != cudaSuccess) return fail(from_cuda(e));
     const int full = per_sm * sm_count(gdev);
     if (o.threads > 0) {
-        p->blocks = (o.threads + block - 1) / block;
+        p->blocks = (o.threads + p->block - 1) / p->block;
     } else {
         p->blocks = full;
     }
@@ -593,6 +593,12 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
         stats->busy_cycles = h[ST_BUSY_CYCLES];
         stats->rounds = h[ST_ROUNDS];
         stats->persistent_threads = p->blocks * p->block;
+#ifdef TQ_AB_PROF
+        fprintf(stderr, "TQPROF idle %.4g prolog %.4g expand %.4g enqueue %.4g | in rounds: col %.4g probe %.4g "
+                "mid %.4g atomic+stage %.4g (SM cycles, summed over warps)\n",
+                (double)h[16], (double)h[17], (double)h[18], (double)h[19], (double)h[20], (double)h[21],
+                (double)(h[18] - h[20] - h[21] - h[22]), (double)h[22]);
+#endif
     }
     if (status == TQ_FINISHED) return TQ_OK;
     if (status == TQ_ABORTED_FULL) return TQ_ERR_QUEUE_FULL;

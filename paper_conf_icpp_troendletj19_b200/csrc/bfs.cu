@@ -32,13 +32,25 @@ namespace tqk {
 
 constexpr int kBlock = 256;          // threads per block (8 warps)
 constexpr int kWarps = kBlock / 32;
-constexpr int kStageCap = 512;       // staged tokens per warp (2 KiB smem)
-constexpr int kU = 4;                // 32-edge rounds in flight per lane
-// Resident blocks per SM requested from ptxas (48 warps/SM; <= 40 registers).
-// The expansion is latency-bound (long-scoreboard stalls on col / mirror /
-// atomicMin); measured on B200 kron24: 6 blocks (40 regs, ~40 B spills) beat
-// 4 blocks (64 regs) by 1.2x and 8 blocks (32 regs, more spills) by 1.07x.
-constexpr int kMinBlocks = 6;
+#ifndef TQ_AB_STAGE
+#define TQ_AB_STAGE 512
+#endif
+constexpr int kStageCap = TQ_AB_STAGE;  // staged tokens per warp (2 KiB smem)
+// A/B builds (scripts/ab_bfs.py) override these with -D; the defaults are
+// the measured best.
+#ifndef TQ_AB_KU
+#define TQ_AB_KU 4
+#endif
+#ifndef TQ_AB_MINB
+#define TQ_AB_MINB 5
+#endif
+constexpr int kU = TQ_AB_KU;         // 32-edge rounds in flight per lane
+// Resident blocks per SM requested from ptxas (40 warps/SM; <= 48 registers).
+// The expansion is bound by the L2 request rate of its random mirror probes
+// (DESIGN.md section 6), so occupancy matters through latency hiding and
+// spills; interleaved A/B on B200 (results/ab_occupancy_r01.md): 5 blocks
+// beat 6 by 1-3% on Kronecker and 8% on the grid, 4 and 8 blocks are slower.
+constexpr int kMinBlocks = TQ_AB_MINB;
 constexpr unsigned kLvlSat = 254;    // byte mirror: 0..253 exact, 254 = ">= 254", 255 = unreached
 // bound on CAS retries of one operation; reaching it can only mean a broken
 // queue state (the loops are lock-free), which is reported as a timeout
@@ -85,6 +97,15 @@ __device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long lon
     asm volatile("ld.global.cg.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
+#ifdef TQ_AB_L1PROBE
+#define ld_cg_u8 ld_ca_u8
+__device__ __forceinline__ unsigned ld_ca_u8(const uint8_t *p, unsigned long long pol)
+{
+    unsigned v;
+    asm volatile("ld.global.ca.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+#endif
 __device__ __forceinline__ unsigned mix32(unsigned x)
 {
     x ^= x >> 16;
@@ -380,6 +401,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     const unsigned lane = threadIdx.x & 31;
     const unsigned warp_gid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     uint32_t *stage = stage_all[threadIdx.x >> 5];
+    // owner lanes of one round's atomicMin candidates (ids go to the stage tail)
+    __shared__ uint8_t cown_all[kWarps][32 * KU];
+    uint8_t *cown = cown_all[threadIdx.x >> 5];
     const tq_device_view q = p.q;
     const unsigned long long cap = q.mask + 1;
     const int chunk = p.chunk;
@@ -432,7 +456,15 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         }
     }
 
+#ifdef TQ_AB_PROF
+#define TQ_PROF_T(v) long long v = clock64()
+#define TQ_PROF_ADD(k, d) do { if (lane == 0) S[16 + (k)] += (unsigned long long)(d); } while (0)
+#else
+#define TQ_PROF_T(v)
+#define TQ_PROF_ADD(k, d)
+#endif
     for (;;) {
+        TQ_PROF_T(t0);
         // ---- Listing 1 + Listing 2: GetWorkToken() ----
         bool got = false, got1 = false;
         uint32_t item = 0;
@@ -463,9 +495,15 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             // lane issues both polls back to back and prefers the chunk
             // (acquire loads: a hit makes the producer's W update visible,
             // with no fence; ld.acquire.gpu is LDG.STRONG.GPU + CCTL.IVALL)
+#ifdef TQ_AB_L1PROBE
+            const unsigned long long sv0 = have ? tq_ld_relaxed(q.slots + (tk & q.mask)) : 0ull;
+            const unsigned long long sv1 =
+                (q1_lane && have1) ? tq_ld_relaxed(q1.slots + (tk1 & q1.mask)) : 0ull;
+#else
             const unsigned long long sv0 = have ? tq_ld_acquire(q.slots + (tk & q.mask)) : 0ull;
             const unsigned long long sv1 =
                 (q1_lane && have1) ? tq_ld_acquire(q1.slots + (tk1 & q1.mask)) : 0ull;
+#endif
             got1 = q1_lane && have1 && (unsigned)sv1 == tk1 + 1u;
             got = !got1 && have && (unsigned)sv0 == tk + 1u;
             item = (uint32_t)((got1 ? sv1 : sv0) >> 32);
@@ -511,11 +549,24 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 backoff = backoff ? min(backoff * 2, (unsigned)p.backoff_ns) : 32u;
                 __nanosleep(backoff);
             }
+            TQ_PROF_ADD(0, clock64() - t0);
             continue;
         }
         backoff = 0;
         idle = 0;
+#ifdef TQ_AB_L1PROBE
+#ifndef TQ_AB_L1REFRESH
+#define TQ_AB_L1REFRESH 63
+#endif
+        if (((++busy) & TQ_AB_L1REFRESH) == 0) {
+            unsigned stv;
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(stv)
+                         : "l"(q.status + (warp_gid % TQ_STATUS_COPIES) * TQ_STATUS_STRIDE) : "memory");
+            if (stv != TQ_RUNNING) break;
+        }
+#else
         if (((++busy) & 63) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
+#endif
         if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY || VARIANT == TQ_VARIANT_AN)
             tq_fence_gpu();  // acquire for the comparators' relaxed dequeues
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
@@ -610,6 +661,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
         }
 
+        TQ_PROF_T(t1);
+        TQ_PROF_ADD(1, t1 - t0);
         // ---- DoWorkUnit(): warp-cooperative expansion ----
         const int deg = (int)(hi - lo);
         const int incl = warp_incl_scan(deg, lane);
@@ -634,10 +687,17 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         // token is found by a 5-step shuffle binary search over the lanes'
         // inclusive prefix sums (a shared-memory prefix-max map was measured
         // and was not faster).
+        const unsigned offer_hi = (unsigned)(offer >> 32);  // BFS: the offered level L + 1
         for (int b = 0; b < total; b += 32 * KU) {
             int32_t u[KU];
-            unsigned long long off[KU];
+            unsigned long long off[KU];  // SSSP: per-edge offer (dist + w, v)
+            unsigned lv1[KU];            // BFS: offered level of each edge's token
+            unsigned ownp = 0;           // BFS: owner lane of edge j in byte j
             bool val[KU];
+#ifdef TQ_AB_PROF
+            long long ta;
+            asm volatile("mov.u64 %0, %%clock64;" : "=l"(ta));
+#endif
 #pragma unroll
             for (int j = 0; j < KU; ++j) {
                 const int g = b + j * 32 + (int)lane;
@@ -645,15 +705,23 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 const int gg = val[j] ? g : total - 1;
                 const int o = owner_of(incl, gg);
                 const long long eb = (long long)tq_shfl64((unsigned long long)ebase, o);
-                off[j] = tq_shfl64(offer, o);
                 u[j] = val[j] ? ld_nc_i32(p.col + eb + gg, pol_stream) : 0;
                 if constexpr (TASK == kTaskSSSP) {
+                    off[j] = tq_shfl64(offer, o);
                     const unsigned wt = val[j] ? (unsigned)ld_nc_i32(p.wgt + eb + gg, pol_stream) : 0u;
                     const unsigned long long d = (off[j] >> 32) + wt;  // dist(v) + w(v -> u)
                     val[j] = val[j] && d < 0xffffffffull;
                     off[j] = (d << 32) | (off[j] & 0xffffffffull);
+                } else {
+                    lv1[j] = __shfl_sync(TQ_FULL_MASK, offer_hi, o);
+                    ownp |= (unsigned)o << (8 * j);
                 }
             }
+#ifdef TQ_AB_PROF
+            long long tb;  // after the col loads returned (the asm consumes them)
+            asm volatile("mov.u64 %0, %%clock64;" : "=l"(tb) : "r"(u[0]), "r"(u[KU - 1]), "r"(u[1]), "r"(u[2]));
+            TQ_PROF_ADD(4, tb - ta);
+#endif
             bool cand[KU];
             if constexpr (TASK == kTaskSSSP) {
                 // prefilter: the packed word itself (dist, parent) -- stale
@@ -665,65 +733,121 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 #pragma unroll
                 for (int j = 0; j < KU; ++j) cand[j] = val[j] && off[j] < w[j];
             } else {
-            // prefilter 1: the byte level mirror (L2-resident; stale values
-            // are never below the true level, R8)
-            unsigned m8[KU];
+                // prefilter 1: the byte level mirror (L2-resident; stale values
+                // are never below the true level, R8)
+                unsigned m8[KU];
 #pragma unroll
-            for (int j = 0; j < KU; ++j) {
-                // offers at level >= 254 cannot be filtered by the saturated
-                // mirror: skip the probe (saves a dependent round trip on deep
-                // graphs, e.g. the grid's 8,191 levels) and go to atomicMin
-                const bool deep = (unsigned)(off[j] >> 32) >= kLvlSat;
-                m8[j] = (val[j] && !deep) ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : kLvlSat;
-            }
-            bool tie[KU];
+                for (int j = 0; j < KU; ++j) {
+                    // offers at level >= 254 cannot be filtered by the saturated
+                    // mirror: skip the probe (saves a dependent round trip on deep
+                    // graphs, e.g. the grid's 8,191 levels) and go to atomicMin
+                    const bool deep = lv1[j] >= kLvlSat;
+                    m8[j] = (val[j] && !deep) ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : kLvlSat;
+                }
+#ifdef TQ_AB_PROF
+                long long tc;  // after the mirror probes returned
+                asm volatile("mov.u64 %0, %%clock64;" : "=l"(tc) : "r"(m8[0]), "r"(m8[KU - 1]), "r"(m8[1]), "r"(m8[2]));
+                TQ_PROF_ADD(5, tc - tb);
+#endif
+                bool tie[KU];
+                bool any_tie = false;
 #pragma unroll
-            for (int j = 0; j < KU; ++j) {
-                const unsigned L1 = (unsigned)(off[j] >> 32);
-                const bool known = m8[j] < kLvlSat;  // exact-or-stale-high level
-                tie[j] = val[j] && min_id && known && m8[j] == L1;
-                cand[j] = val[j] && !(known && m8[j] <= L1);
-            }
-            // prefilter 2 (min-id parents only): the packed word, only for
-            // offers that tie on level and may still win on parent id
-            bool any_tie = false;
+                for (int j = 0; j < KU; ++j) {
+                    const bool known = m8[j] < kLvlSat;  // exact-or-stale-high level
+                    tie[j] = val[j] && min_id && known && m8[j] == lv1[j];
+                    cand[j] = val[j] && !(known && m8[j] <= lv1[j]);
+                    any_tie |= tie[j];
+                }
+                // prefilter 2 (min-id parents only): the packed word, only for
+                // offers that tie on level and may still win on parent id
+                if (min_id && __any_sync(TQ_FULL_MASK, any_tie)) {
+                    unsigned long long w[KU];
 #pragma unroll
-            for (int j = 0; j < KU; ++j) any_tie |= tie[j];
-            if (min_id && __any_sync(TQ_FULL_MASK, any_tie)) {
-                unsigned long long w[KU];
+                    for (int j = 0; j < KU; ++j) w[j] = tie[j] ? ld_cg_u64(p.W + u[j]) : 0ull;
 #pragma unroll
-                for (int j = 0; j < KU; ++j) w[j] = tie[j] ? ld_cg_u64(p.W + u[j]) : 0ull;
-#pragma unroll
-                for (int j = 0; j < KU; ++j) cand[j] = cand[j] || (tie[j] && off[j] < w[j]);
-            }
-            }
-            bool nt[KU];
-            unsigned n_min = 0, n_reenq = 0;
-#pragma unroll
-            for (int j = 0; j < KU; ++j) {
-                nt[j] = false;
-                bool re = false;
-                if (cand[j]) {
-                    const unsigned long long old = atomicMin(p.W + u[j], off[j]);
-                    const unsigned L1 = (unsigned)(off[j] >> 32);
-                    if ((old >> 32) > L1) {  // level strictly lowered: (re)discovered
-                        nt[j] = true;
-                        if constexpr (TASK == kTaskBFS) st_u8(p.lvl8 + u[j], L1 < kLvlSat ? L1 : kLvlSat);
-                        re = (old >> 32) != 0xffffffffull;
+                    for (int j = 0; j < KU; ++j) {
+                        const unsigned long long oj = tq_shfl64(offer, (ownp >> (8 * j)) & 31u);
+                        cand[j] = cand[j] || (tie[j] && oj < w[j]);
                     }
                 }
-                n_min += __popc(__ballot_sync(TQ_FULL_MASK, cand[j]));
-                n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, re));
             }
-            if (lane == 0) {
-                S[ST_MIN_ATOMICS] += n_min;
-                S[ST_REENQUEUES] += n_reenq;
-            }
+#ifdef TQ_AB_PROF
+            long long td;
+            asm volatile("mov.u64 %0, %%clock64;" : "=l"(td));
+#endif
+            if constexpr (TASK == kTaskBFS) {
+                // Candidates (a few percent of the edges) are compacted into
+                // the free tail of the staging buffer -- vertex ids at
+                // stage[cnt..), owner lanes in cown[] -- and their atomicMins
+                // issued as dense warp instructions, so the round trips of a
+                // round's atomics overlap instead of running one per j (the
+                // mirror stores between them are ordered).  The vertices whose
+                // level fell are then compacted in place, to stage[cnt..).
+                unsigned ncand = 0;
 #pragma unroll
-            for (int j = 0; j < KU; ++j) {
-                const unsigned m = __ballot_sync(TQ_FULL_MASK, nt[j]);
-                if (nt[j]) stage[cnt + __popc(m & tq_lanemask_lt())] = (uint32_t)u[j];
-                cnt += __popc(m);
+                for (int j = 0; j < KU; ++j) {
+                    const unsigned m = __ballot_sync(TQ_FULL_MASK, cand[j]);
+                    if (cand[j]) {
+                        const unsigned k = ncand + __popc(m & tq_lanemask_lt());
+                        stage[cnt + k] = (uint32_t)u[j];
+                        cown[k] = (uint8_t)(ownp >> (8 * j));
+                    }
+                    ncand += __popc(m);
+                }
+                if (ncand) {
+                    __syncwarp();
+                    unsigned n_reenq = 0, wr = cnt;
+                    for (unsigned i0 = 0; i0 < ncand; i0 += 32) {
+                        const unsigned i = i0 + lane;
+                        const bool c = i < ncand;
+                        const uint32_t cv = c ? stage[cnt + i] : 0u;
+                        const unsigned long long co = tq_shfl64(offer, c ? cown[i] : 0u);
+                        __syncwarp();  // all reads of this slice before the in-place writes
+                        const unsigned L1 = (unsigned)(co >> 32);
+                        const unsigned oldhi = c ? (unsigned)(atomicMin(p.W + cv, co) >> 32) : 0u;
+                        const bool nt = c && oldhi > L1;  // level strictly lowered: (re)discovered
+                        if (nt) st_u8(p.lvl8 + cv, L1 < kLvlSat ? L1 : kLvlSat);
+                        n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, nt && oldhi != 0xffffffffu));
+                        const unsigned m = __ballot_sync(TQ_FULL_MASK, nt);
+                        if (nt) stage[wr + __popc(m & tq_lanemask_lt())] = cv;
+                        wr += __popc(m);
+                        __syncwarp();
+                    }
+                    cnt = wr;
+                    if (lane == 0) {
+                        S[ST_MIN_ATOMICS] += ncand;
+                        S[ST_REENQUEUES] += n_reenq;
+                    }
+                }
+            } else {
+                bool nt[KU];
+                unsigned n_min = 0, n_reenq = 0;
+#pragma unroll
+                for (int j = 0; j < KU; ++j) {
+                    nt[j] = false;
+                    bool re = false;
+                    if (cand[j]) {
+                        const unsigned long long old = atomicMin(p.W + u[j], off[j]);
+                        const unsigned L1 = (unsigned)(off[j] >> 32);
+                        if ((old >> 32) > L1) {  // level strictly lowered: (re)discovered
+                            nt[j] = true;
+                            if constexpr (TASK == kTaskBFS) st_u8(p.lvl8 + u[j], L1 < kLvlSat ? L1 : kLvlSat);
+                            re = (old >> 32) != 0xffffffffull;
+                        }
+                    }
+                    n_min += __popc(__ballot_sync(TQ_FULL_MASK, cand[j]));
+                    n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, re));
+                }
+                if (lane == 0) {
+                    S[ST_MIN_ATOMICS] += n_min;
+                    S[ST_REENQUEUES] += n_reenq;
+                }
+#pragma unroll
+                for (int j = 0; j < KU; ++j) {
+                    const unsigned m = __ballot_sync(TQ_FULL_MASK, nt[j]);
+                    if (nt[j]) stage[cnt + __popc(m & tq_lanemask_lt())] = (uint32_t)u[j];
+                    cnt += __popc(m);
+                }
             }
             if (cnt > kStageCap - 32 * KU) {
                 __syncwarp();
@@ -731,8 +855,17 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 __syncwarp();
                 cnt = 0;
             }
+#ifdef TQ_AB_PROF
+            {
+                long long te;
+                asm volatile("mov.u64 %0, %%clock64;" : "=l"(te));
+                TQ_PROF_ADD(6, te - td);  // atomics + staging (+ flushes)
+            }
+#endif
         }
 
+        TQ_PROF_T(t2);
+        TQ_PROF_ADD(2, t2 - t1);
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
         enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
@@ -771,6 +904,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 ++st_qatom;
             }
         }
+        TQ_PROF_ADD(3, clock64() - t2);
     }
 
     // ---- statistics (one atomic per counter per warp) ----
@@ -783,6 +917,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         }
         __syncwarp();
         if (lane < ST_REACHED && S[lane]) atomicAdd(p.stats + lane, S[lane]);
+#ifdef TQ_AB_PROF
+        if (lane >= 16 && lane < 23) atomicAdd(p.stats + lane, S[lane]);
+#endif
     }
 }
 

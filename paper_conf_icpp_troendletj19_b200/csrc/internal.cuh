@@ -29,7 +29,11 @@ __device__ __forceinline__ unsigned long long *per_lane_addr(unsigned long long 
     return p + (tq_lane() & zero);
 }
 
+#ifdef TQ_AB_PROF
+constexpr int kStatCount = 24;  // 16..19: idle / prolog / expand / enqueue SM cycles (A/B builds only)
+#else
 constexpr int kStatCount = 16;
+#endif
 
 // Task run by the persistent kernel over the queue (the queue is the same).
 constexpr int kTaskBFS = 0;   // top-down BFS levels (the paper's driver)
