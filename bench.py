@@ -195,6 +195,10 @@ def main():
         return plan.run(r, level, parent, grow_on_full=True)
 
     multiroot.run_local(run_root, mine, steps=args.warmup)
+    # the expansion's second ceiling, measured live on this GPU (outside the
+    # timed region): random 1-byte L2 probes over a table the size of the
+    # level mirror, at the persistent kernel's shape
+    probe_g = tq.probe_ceiling(max(n, 1 << 12), 1 << 28, device=local) if kind == "kron" else None
 
     # ---- timed region: K steps, barrier + sync on both sides, device events ----
     if dist:
@@ -231,6 +235,16 @@ def main():
     tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+
+    probe_roof = None
+    if probe_g:
+        scanned = agg["edges_scanned"] / runs_all
+        probe_roof = {"bound": "l2_random_probe", "achieved": round(scanned / avg_kernel_s / 1e9, 1),
+                      "peak": round(probe_g, 1), "unit": "G probes/s",
+                      "frac": round(scanned / avg_kernel_s / 1e9 / probe_g, 4),
+                      "what": "CSR entries scanned per second of the persistent kernel (one random "
+                              "32 B L2 sector each: the level-mirror probe) vs tq_probe_ceiling over a "
+                              "table of the mirror's size, measured in this run"}
 
     # ---- e2e through the public API with host buffers (pinned), every step ----
     e2e = None
@@ -312,6 +326,7 @@ def main():
                          "kernel": "bfs_persistent_kernel<RF_AN>", "peak_source": peak_src,
                          "alg_bytes_per_launch": int(alg_bytes),
                          "avg_launch_ms": round(avg_kernel_s * 1e3, 4)},
+            "roofline_l2_probe": probe_roof,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,

@@ -301,6 +301,19 @@ const char *tq_version(void);
  * an unknown name: lets bindings check their struct mirrors without a GPU. */
 size_t tq_struct_size(const char *name);
 
+/* Measurement utility (the roofline of the BFS
+ * expansion): the random-probe ceiling of this GPU.  Streams `probes` 4-byte
+ * indices (uniform random over [0, table_bytes), generated on the device) and
+ * reads one byte of a table_bytes-long table per index with ld.global.cg (L2),
+ * 4 probes in flight per lane, at the BFS kernel's shape (256-thread blocks,
+ * its occupancy): the access pattern of the expansion's level-mirror probes
+ * (one random 32-byte sector per CSR entry).  *g_per_s = probes per second /
+ * 1e9 of the second of two launches (CUDA events on `stream`).  Allocates and
+ * frees its own device memory.  table_bytes in [2^12, 2^32), probes in
+ * [2^20, 2^32); TQ_ERR_INVALID otherwise.  Synchronous. */
+tq_status tq_probe_ceiling(int device, uint64_t table_bytes, uint64_t probes, void *stream,
+                           double *g_per_s);
+
 #ifdef __cplusplus
 }
 #endif

@@ -94,6 +94,7 @@ EXPORTS = {
                                              ctypes.POINTER(ctypes.c_int)]),
     "tq_version": (ctypes.c_char_p, []),
     "tq_struct_size": (ctypes.c_size_t, [ctypes.c_char_p]),
+    "tq_probe_ceiling": (ctypes.c_int, [ctypes.c_int, c_u64, c_u64, c_vp, ctypes.POINTER(c_dbl)]),
 }
 
 STRUCTS = {"tq_csr": tq_csr, "bfs_opts": bfs_opts, "bfs_stats": bfs_stats, "tq_device_view": tq_device_view,

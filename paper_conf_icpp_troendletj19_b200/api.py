@@ -347,5 +347,14 @@ def persistent_threads(variant="rf_an", device: int = 0) -> int:
     return t.value
 
 
+def probe_ceiling(table_bytes: int, probes: int = 1 << 28, device: int = 0, stream=None) -> float:
+    """G random L2 byte probes per second on this GPU (tq_probe_ceiling): the
+    ceiling of the BFS expansion's mirror probes."""
+    g = ctypes.c_double()
+    check(lib().tq_probe_ceiling(int(device), int(table_bytes), int(probes), _stream_ptr(stream),
+                                 ctypes.byref(g)), "tq_probe_ceiling")
+    return g.value
+
+
 def version() -> str:
     return lib().tq_version().decode()

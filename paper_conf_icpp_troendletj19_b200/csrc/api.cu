@@ -753,6 +753,20 @@ tq_status sssp_run_ex(const tq_csr *g, const int32_t *weights, int32_t src, uint
 // ------------------------------------------------------------------------
 // queue micro-benchmark
 // ------------------------------------------------------------------------
+tq_status tq_probe_ceiling(int device, uint64_t table_bytes, uint64_t probes, void *stream, double *g_per_s)
+{
+    if (!g_per_s || table_bytes < (1ull << 12) || table_bytes >= (1ull << 32) || probes < (1ull << 20) ||
+        probes >= (1ull << 32))
+        return TQ_ERR_INVALID;
+    *g_per_s = 0.0;
+    DeviceGuard g(device);
+    if (!g.ok) return TQ_ERR_INVALID;
+    int per_sm = 0;  // the BFS kernel's occupancy: same block shape, same residency
+    CK(bfs_occupancy(TQ_VARIANT_RF_AN, 256, &per_sm));
+    CK(probe_ceiling(table_bytes, probes, per_sm, (cudaStream_t)stream, g_per_s));
+    return TQ_OK;
+}
+
 tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
 {
     if (!c || !r) return TQ_ERR_INVALID;

@@ -377,6 +377,79 @@ cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int bloc
     }
 }
 
+// ---------------------------------------------------------------------------
+// Random-probe ceiling (tq_probe_ceiling): the expansion's mirror-probe access
+// pattern alone -- a coalesced 4-byte index stream and one random byte probe
+// per index through L2, 4 in flight per lane, the BFS kernel's block shape.
+// ---------------------------------------------------------------------------
+__global__ void probe_fill_kernel(uint32_t *idx, unsigned long long n, unsigned long long range,
+                                  unsigned long long seed)
+{
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        unsigned long long x = (i + 1) * 0x9E3779B97F4A7C15ull ^ seed;  // splitmix64 finaliser
+        x ^= x >> 31;
+        x *= 0xBF58476D1CE4E5B9ull;
+        x ^= x >> 29;
+        idx[i] = (uint32_t)(x % range);
+    }
+}
+
+__global__ void __launch_bounds__(256) probe_ceiling_kernel(const uint32_t *idx, unsigned long long n,
+                                                            const uint8_t *tab, unsigned long long *sink)
+{
+    const unsigned long long tid = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    unsigned acc = 0;
+    for (unsigned long long i = tid; i < n; i += 4 * stride) {
+        uint32_t u[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) u[j] = (i + j * stride < n) ? __ldg(idx + i + j * stride) : 0u;
+        unsigned m[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) asm volatile("ld.global.cg.u8 %0, [%1];" : "=r"(m[j]) : "l"(tab + u[j]));
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc += m[j];
+    }
+    if (acc == 0xdeadbeefu) *sink = acc;  // keeps the probes live
+}
+
+cudaError_t probe_ceiling(unsigned long long table_bytes, unsigned long long probes, int blocks_per_sm,
+                          cudaStream_t s, double *g_per_s)
+{
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    uint32_t *idx = nullptr;
+    uint8_t *tab = nullptr;
+    unsigned long long *sink = nullptr;
+    cudaEvent_t a = nullptr, b = nullptr;
+    cudaError_t e = cudaMalloc(&idx, probes * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&tab, table_bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&sink, 8);
+    if (e == cudaSuccess) e = cudaMemsetAsync(tab, 1, table_bytes, s);
+    if (e == cudaSuccess) e = cudaEventCreate(&a);
+    if (e == cudaSuccess) e = cudaEventCreate(&b);
+    if (e == cudaSuccess) {
+        probe_fill_kernel<<<sms * 8, 256, 0, s>>>(idx, probes, table_bytes, 12345ull);
+        probe_ceiling_kernel<<<sms * blocks_per_sm, 256, 0, s>>>(idx, probes, tab, sink);  // warm-up
+        cudaEventRecord(a, s);
+        probe_ceiling_kernel<<<sms * blocks_per_sm, 256, 0, s>>>(idx, probes, tab, sink);
+        cudaEventRecord(b, s);
+        e = cudaEventSynchronize(b);
+        if (e == cudaSuccess) e = cudaGetLastError();
+        float ms = 0;
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, a, b);
+        if (e == cudaSuccess) *g_per_s = (double)probes / (ms * 1e-3) / 1e9;
+    }
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+    cudaFree(idx);
+    cudaFree(tab);
+    cudaFree(sink);
+    return e;
+}
+
 cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm)
 {
     switch (variant) {

@@ -109,5 +109,7 @@ struct BenchParams {
 };
 cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int block, cudaStream_t s);
 cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm);
+cudaError_t probe_ceiling(unsigned long long table_bytes, unsigned long long probes, int blocks_per_sm,
+                          cudaStream_t s, double *g_per_s);
 
 }  // namespace tqk

@@ -11,7 +11,7 @@ from __future__ import annotations
 
 from typing import Callable, Sequence
 
-STAT_KEYS = ("ms", "traversed_edges", "reached", "ms_kernel", "launches", "runs")
+STAT_KEYS = ("ms", "traversed_edges", "reached", "ms_kernel", "launches", "runs", "edges_scanned")
 
 
 def split_roots(roots: Sequence[int], rank: int, world: int) -> list[int]:
@@ -35,7 +35,8 @@ def local_vector(stats: list[dict], ms_total: float, launches_per_run: int = 3):
     """Per-rank summary in STAT_KEYS order."""
     return [float(ms_total), float(sum(s["traversed_edges"] for s in stats)),
             float(sum(s["reached"] for s in stats)), float(sum(s.get("ms_kernel", 0.0) for s in stats)),
-            float(launches_per_run * len(stats)), float(len(stats))]
+            float(launches_per_run * len(stats)), float(len(stats)),
+            float(sum(s.get("edges_scanned", 0) for s in stats))]
 
 
 def gather(vec, dist=None, device=None):

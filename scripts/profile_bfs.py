@@ -23,7 +23,7 @@ plan = tq.BfsPlan(rp, col, variant=args.variant)
 lv = torch.empty(n, dtype=torch.int32, device=dev)
 pa = torch.empty(n, dtype=torch.int32, device=dev)
 for i in range(args.runs):
-    st = plan.run(roots[0], lv, pa)
+    st = plan.run(roots[0], lv, pa, grow_on_full=True)
     print({k: st[k] for k in ("ms", "ms_kernel", "traversed_edges", "reached", "tasks", "chunk_tasks",
                               "edges_scanned", "min_atomics", "reenqueues", "queue_atomics",
                               "empty_polls", "max_level")})

@@ -15,7 +15,7 @@ import paper_conf_icpp_troendletj19_b200 as tq
 ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="kron24x8")
 ap.add_argument("--roots", type=int, default=4)
-ap.add_argument("--mode", default="sorted", choices=["sorted", "strided"])
+ap.add_argument("--mode", default="sorted", choices=["sorted", "strided", "compact"])
 ap.add_argument("--hub-shift", type=int, default=7)
 ap.add_argument("--hubs", type=int, default=1 << 17)
 ap.add_argument("--cache", type=int, default=1, help="strided: enable the hub level cache")
@@ -30,6 +30,20 @@ if args.mode == "sorted":
     new2old = torch.sort(deg, descending=True, stable=True).indices
     old2new = torch.empty_like(new2old)
     old2new[new2old] = torch.arange(n, device=dev)
+elif args.mode == "compact":  # top-H degree vertices moved to ids 0..H-1 (swaps), the rest unchanged
+    H = args.hubs
+    top = torch.sort(deg, descending=True, stable=True).indices[:H]
+    is_hub = torch.zeros(n, dtype=torch.bool, device=dev)
+    is_hub[top] = True
+    is_slot = torch.zeros(n, dtype=torch.bool, device=dev)
+    is_slot[:H] = True
+    A = torch.nonzero(is_hub & ~is_slot).flatten()
+    B = torch.nonzero(is_slot & ~is_hub).flatten()
+    new2old = torch.arange(n, device=dev)
+    new2old[A] = B
+    new2old[B] = A
+    old2new = new2old
+    print("hubs", H, "moved", A.numel(), "hub edge share %.3f" % (float(deg[top].sum()) / float(deg.sum())))
 else:  # top-H degree vertices moved to ids k << shift (swaps), the rest unchanged
     S = 1 << args.hub_shift
     H = min(args.hubs, (n + S - 1) // S)
