@@ -263,14 +263,19 @@ def main():
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
         te_e2e = 0
+        step_s = []
         for _ in range(args.steps):
+            ts0 = time.perf_counter()
             with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=stream, device=local,
                             parents=args.parents) as hp:
+                ts1 = time.perf_counter()  # bfs_plan_create returns after the H2D copies
                 # one C-ABI call per step: every root's level and parent arrays
                 # are copied to the (reused) pinned host buffers, D2H overlapped
                 # with the next root's BFS on a second stream
                 for s in hp.run_batch(mine, lv_np, pa_np, stride=0):
                     te_e2e += s["traversed_edges"]
+                ts2 = time.perf_counter()
+            step_s.append([round(ts1 - ts0, 3), round(ts2 - ts1, 3), round(time.perf_counter() - ts2, 3)])
         torch.cuda.synchronize(dev)
         sec = time.perf_counter() - t0
         secv = torch.tensor([sec, te_e2e], dtype=torch.float64, device=dev)
@@ -284,6 +289,7 @@ def main():
         e2e = {"value": te_tot / sec_max / 1e9, "unit": "GTEPS",
                "h2d_bytes_per_step": int((n + 1) * 8 + col.numel() * 4),
                "d2h_bytes_per_step": int(len(mine) * n * 8),
+               "step_s_create_batch_destroy": step_s,
                "timed": "host perf_counter per step around bfs_plan_create(pinned host CSR: H2D) + "
                         "bfs_plan_run_batch(all roots, pinned host level/parent: D2H per root), synchronised"}
 

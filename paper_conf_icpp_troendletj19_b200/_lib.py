@@ -119,6 +119,8 @@ def lib() -> ctypes.CDLL:
                 "(nvcc, sm_100a). There is no CPU fallback.")
         L = ctypes.CDLL(LIB_PATH)
         for name, (res, args) in EXPORTS.items():
+            if os.environ.get("TQ_LIB") and not hasattr(L, name):
+                continue  # A/B runs of an older build: entry points it predates stay unbound
             f = getattr(L, name)
             f.restype = res
             f.argtypes = args

@@ -529,6 +529,10 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.l2_window_bytes = p->l2_window;
     bp.delay_ns = (unsigned)p->delay_ns;
     bp.delay_seed = p->delay_seed;
+    // every slot of [t0, t0 + C) holds "empty for t" when a run starts (after
+    // a reset, or at Rear after a finished run; see plan_finish)
+    bp.q_lap_end = p->next_ticket + (bp.q.mask + 1);
+    bp.q1_lap_end = p->hub_queue ? p->next_ticket1 + (bp.q1.mask + 1) : 0ull;
 
     CK(cudaEventRecord(p->ev[0], s));
     CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));

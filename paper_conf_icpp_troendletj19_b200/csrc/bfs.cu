@@ -307,10 +307,15 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
 // Enqueue of a warp's staged tokens (Listing 3).  `items` in shared memory,
 // `cnt` warp-uniform.  Coalesced: lane i writes tickets base+i, base+i+32, ...
 // ---------------------------------------------------------------------------
+//
+// lap_end: every slot of a ticket below lap_end is known to hold "empty for
+// t" -- at run start all slots of [t0, t0 + C) do (R18) -- so
+// Listing 3's queue-full check (P:268 line 25) cannot fail there and its slot
+// read is skipped; tickets at or past lap_end are checked.
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const uint32_t *items,
                                                unsigned cnt, unsigned lane, unsigned *qatom,
-                                               unsigned *casfail)
+                                               unsigned *casfail, unsigned long long lap_end)
 {
     if (cnt == 0) return;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
@@ -323,6 +328,13 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
         // release: the W updates (and this warp's Rear reservation) are
         // ordered before the tokens that name them
         tq_fence_release();
+        if (VARIANT == TQ_VARIANT_RF_AN && base + cnt <= lap_end) {  // warp-uniform
+            for (unsigned i = lane; i < cnt; i += 32) {
+                const unsigned long long t = base + i;
+                tq_st_relaxed(q.slots + (t & q.mask), ((unsigned long long)items[i] << 32) | (unsigned)(t + 1));
+            }
+            return;
+        }
         for (unsigned i0 = 0; i0 < cnt; i0 += 32 * 4) {
             unsigned long long sv[4];
 #pragma unroll
@@ -364,7 +376,8 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
 // chunk tokens of one hub: CHUNK_FLAG | (first + k), k < n (warp-uniform args)
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t first, unsigned n,
-                                               unsigned lane, unsigned *qatom, unsigned *casfail)
+                                               unsigned lane, unsigned *qatom, unsigned *casfail,
+                                               unsigned long long lap_end)
 {
     if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
         for (unsigned i = lane; i < n; i += 32)
@@ -385,6 +398,12 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
             }
             for (unsigned k = 0; k < mine; ++k)
                 tq_publish(q, base + k, CHUNK_FLAG | (first + lane + 32 * k));
+            return;
+        }
+        if (VARIANT == TQ_VARIANT_RF_AN && base + n <= lap_end) {  // first lap: no full check
+            for (unsigned i = lane; i < n; i += 32)
+                tq_st_relaxed(q.slots + ((base + i) & q.mask),
+                              ((unsigned long long)(CHUNK_FLAG | (first + i)) << 32) | (unsigned)(base + i + 1));
             return;
         }
         for (unsigned i = lane; i < n; i += 32) tq_publish(q, base + i, CHUNK_FLAG | (first + i));
@@ -851,7 +870,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
             if (cnt > kStageCap - 32 * KU) {
                 __syncwarp();
-                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
+                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end);
                 __syncwarp();
                 cnt = 0;
             }
@@ -868,7 +887,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         TQ_PROF_ADD(2, t2 - t1);
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
-        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail);
+        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end);
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
         const bool hubm_any = hubm != 0;
@@ -877,7 +896,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             hubm &= hubm - 1;
             const unsigned n = __shfl_sync(TQ_FULL_MASK, nch, h);
             const uint32_t first = __shfl_sync(TQ_FULL_MASK, chb, h);
-            enqueue_chunks<VARIANT>(hubq ? q1 : q, first, n, lane, &st_qatom, &st_fail);
+            enqueue_chunks<VARIANT>(hubq ? q1 : q, first, n, lane, &st_qatom, &st_fail,
+                                    hubq ? p.q1_lap_end : p.q_lap_end);
         }
 
         // ---- completion accounting for WorkRemains() (R6) ----

@@ -82,6 +82,10 @@ struct BfsParams {
     size_t l2_window_bytes;    // persisting-L2 window over lvl8 (0 = none)
     unsigned delay_ns;         // test only: schedule perturbation (bfs_opts.debug_delay_ns)
     unsigned delay_seed;
+    // first-lap bounds: tickets below these are known empty at run start
+    // (t0 + C of each queue), so their enqueue skips the full check
+    unsigned long long q_lap_end;
+    unsigned long long q1_lap_end;
 };
 
 // bfs.cu
