@@ -1,5 +1,5 @@
 import json, sys, os
-sys.path.insert(0, os.getcwd())
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_icpp_troendletj19_b200 as tq
 full = tq.queue_bench("rf_an", warps=0, batch=32, items=1 << 22)["warps"]
 for v in ("rf_an", "rf_an_cta"):

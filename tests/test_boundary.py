@@ -108,3 +108,14 @@ def test_missing_library_fails_loudly(monkeypatch, tmp_path):
 def test_input_generator_builds():
     import inputs.gpu
     assert os.path.exists(inputs.gpu.build())
+
+
+def test_probe_ceiling_rejects_bad_sizes(libtq):
+    """Argument checks run before any device work (no GPU needed)."""
+    import ctypes
+    from paper_conf_icpp_troendletj19_b200 import _lib
+    L = _lib.lib()
+    g = ctypes.c_double(-1.0)
+    for table, probes in [(1 << 11, 1 << 22), (1 << 32, 1 << 22), (1 << 20, 1 << 19), (1 << 20, 1 << 32)]:
+        assert L.tq_probe_ceiling(0, table, probes, None, ctypes.byref(g)) == -1
+    assert L.tq_probe_ceiling(0, 1 << 20, 1 << 22, None, None) == -1

@@ -335,3 +335,26 @@ def test_any_parent_rule_levels_exact_tree_valid(tq, variant):
         reached = lv_o > 0
         assert np.all(lv_o[pa[reached]] == lv_o[reached] - 1)
         assert st["traversed_edges"] == info["traversed_edges"]
+
+
+def test_ring_wraps_within_runs(tq):
+    """A queue smaller than one run's ticket count: every run crosses the
+    first-lap boundary t0 + C (R18) and the ring wraps many times
+    across consecutive runs on one plan; results stay exact."""
+    import torch
+    g = kronecker_csr(10, 16, 1)
+    rp, col = to_dev(g)
+    level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+    parent = torch.empty_like(level)
+    with tq.BfsPlan(rp, col, capacity=1024, parents="min_id") as plan:
+        tickets = 0
+        for r in sample_roots(g.row_ptr, 12, 5):
+            st = plan.run(int(r), level, parent, grow_on_full=True)
+            tickets += st["tickets"]
+            check_against_oracle(g, int(r), level, parent, st, min_id=True)
+    assert tickets > 8 * 1024
+
+
+def test_probe_ceiling_measures(tq):
+    g = tq.probe_ceiling(1 << 24, 1 << 22)
+    assert 1.0 < g < 10000.0
