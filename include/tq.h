@@ -58,10 +58,14 @@ typedef enum {
                                       reserving n slots)             */
     TQ_VARIANT_ATOMIC_CEILING = 4, /* tq_bench only: proxy atomicAdd on Rear
                                       with no slot traffic -> R_atom          */
-    TQ_VARIANT_RF_AN_CTA = 5       /* tq_bench only: RF/AN with the CTA as the
+    TQ_VARIANT_RF_AN_CTA = 5,      /* tq_bench only: RF/AN with the CTA as the
                                       proxy group (one atomicAdd on Rear and
                                       one on Front per block per iteration;
                                       the abstract's "thread group")   */
+    TQ_VARIANT_RF_AN_CLUSTER = 6   /* tq_bench only, pipelined (depth 2): RF/AN
+                                      with a thread-block cluster of
+                                      cfg.cluster CTAs as the proxy group
+                                      (bases broadcast over DSMEM)           */
 } tq_variant;
 
 /* ------------------------------------------------------------------------ */
@@ -271,6 +275,16 @@ typedef struct {
     void *stream;
     double timeout_s;   /* 0 = 60 s                                           */
     int device;
+    int depth;          /* 0/1: per iteration reserve Rear, publish, reserve
+                           Front, poll (the paper's order).  2: pipelined --
+                           the proxy reserves iteration k+1's Rear and Front
+                           tickets at the start of iteration k and publishes
+                           k+1's items after k's poll (<= 2b items in flight
+                           per warp; RF_AN_CTA and RF_AN_CLUSTER only, else
+                           TQ_ERR_UNSUPPORTED)                               */
+    int cluster;        /* RF_AN_CLUSTER: CTAs per cluster (0 = 4; 1..16);
+                           warps must be a multiple of 8*cluster and fit the
+                           co-resident cluster count, else TQ_ERR_INVALID    */
 } tq_bench_cfg;
 
 typedef struct {

@@ -17,7 +17,8 @@ c_i32, c_i64, c_u32, c_u64, c_dbl, c_vp = (ctypes.c_int32, ctypes.c_int64, ctype
 TQ_OK, TQ_ERR_INVALID, TQ_ERR_CUDA, TQ_ERR_NOMEM, TQ_ERR_QUEUE_FULL, TQ_ERR_TIMEOUT, \
     TQ_ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 
-VARIANTS = {"rf_an": 0, "per_thread_afa": 1, "cas_retry": 2, "an": 3, "atomic_ceiling": 4, "rf_an_cta": 5}
+VARIANTS = {"rf_an": 0, "per_thread_afa": 1, "cas_retry": 2, "an": 3, "atomic_ceiling": 4, "rf_an_cta": 5,
+            "rf_an_cluster": 6}
 STATUS_NAMES = {0: "running", 1: "finished", 2: "aborted_full", 3: "aborted_timeout"}
 PARENT_RULES = {"any": 0, "min_id": 1}
 
@@ -56,7 +57,8 @@ class tq_bench_cfg(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int), ("warps", ctypes.c_int), ("batch", ctypes.c_int),
                 ("items", c_u64), ("capacity", c_u64), ("work_iters", ctypes.c_int), ("seed", c_u64),
                 ("log_mode", ctypes.c_int), ("enq_log", c_vp), ("deq_log", c_vp), ("stream", c_vp),
-                ("timeout_s", c_dbl), ("device", ctypes.c_int)]
+                ("timeout_s", c_dbl), ("device", ctypes.c_int), ("depth", ctypes.c_int),
+                ("cluster", ctypes.c_int)]
 
 
 class tq_bench_result(ctypes.Structure):

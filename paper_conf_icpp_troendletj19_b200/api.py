@@ -316,9 +316,12 @@ class Queue:
 
 def queue_bench(variant="rf_an", *, warps: int = 0, batch: int = 32, items: int = 1 << 24,
                 capacity: int = 1 << 20, work_iters: int = 0, seed: int = 3, log: bool = False,
-                stream=None, timeout_s: float = 0.0, device: int = 0) -> dict:
+                stream=None, timeout_s: float = 0.0, device: int = 0, depth: int = 1,
+                cluster: int = 0) -> dict:
     """`tq_bench`: enqueue/dequeue throughput of one queue variant.
 
+    depth=2 pipelines one iteration ahead (rf_an, rf_an_cta; rf_an_cluster
+    always); cluster = CTAs per proxy group of rf_an_cluster (0 -> 4).
     With log=True returns 'enq_log' / 'deq_log' (ticket -> item, CUDA tensors).
     """
     enq_log = deq_log = None
@@ -328,7 +331,7 @@ def queue_bench(variant="rf_an", *, warps: int = 0, batch: int = 32, items: int 
         deq_log = torch.zeros(items, dtype=torch.int32, device=f"cuda:{device}")
     cfg = _lib.tq_bench_cfg(_variant(variant), int(warps), int(batch), int(items), int(capacity),
                             int(work_iters), int(seed), int(log), _ptr(enq_log), _ptr(deq_log),
-                            _stream_ptr(stream), float(timeout_s), int(device))
+                            _stream_ptr(stream), float(timeout_s), int(device), int(depth), int(cluster))
     res = _lib.tq_bench_result()
     status = lib().tq_bench(ctypes.byref(cfg), ctypes.byref(res))
     out = {f: getattr(res, f) for f, _ in res._fields_}

@@ -775,14 +775,28 @@ tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
 {
     if (!c || !r) return TQ_ERR_INVALID;
     memset(r, 0, sizeof(*r));
-    if (c->variant < TQ_VARIANT_RF_AN || c->variant > TQ_VARIANT_RF_AN_CTA) return TQ_ERR_UNSUPPORTED;
+    if (c->variant < TQ_VARIANT_RF_AN || c->variant > TQ_VARIANT_RF_AN_CLUSTER) return TQ_ERR_UNSUPPORTED;
     if (c->batch < 1 || c->batch > 32 || c->items == 0 || c->warps < 0) return TQ_ERR_INVALID;
+    if (c->depth < 0 || c->depth > 2) return TQ_ERR_INVALID;
+    const bool cluster_v = c->variant == TQ_VARIANT_RF_AN_CLUSTER;
+    const int depth = cluster_v ? 2 : (c->depth == 0 ? 1 : c->depth);
+    if (depth == 2 && c->variant != TQ_VARIANT_RF_AN_CTA && !cluster_v) return TQ_ERR_UNSUPPORTED;
+    const int csize = cluster_v ? (c->cluster == 0 ? 4 : c->cluster) : 1;
+    if (csize < 1 || csize > 16) return TQ_ERR_INVALID;
     DeviceGuard g(c->device);
     if (!g.ok) return TQ_ERR_INVALID;
     int warps = c->warps;
-    if (warps == 0) {
+    if (cluster_v) {
+        int clusters = 0;
+        CK(bench_max_clusters(csize, 256, &clusters));
+        if (warps == 0) warps = clusters * csize * 8;
+        if (warps % (8 * csize) || warps > clusters * csize * 8 || warps == 0) return TQ_ERR_INVALID;
+    } else if (warps == 0) {
         int per_sm = 0;
-        CK(bench_occupancy(c->variant, 256, &per_sm));
+        if (depth == 2)
+            CK(bench_pipe_occupancy(256, &per_sm));
+        else
+            CK(bench_occupancy(c->variant, 256, &per_sm));
         warps = per_sm * sm_count(c->device) * 8;
     }
     int wpb = 8;
@@ -793,7 +807,8 @@ tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
     const uint64_t items = iters * warps * c->batch;
     if (c->log_mode && (!c->enq_log || !c->deq_log)) return TQ_ERR_INVALID;
     uint64_t cap = c->capacity ? c->capacity : (1ull << 20);
-    if ((uint64_t)warps * c->batch > next_pow2(cap)) return TQ_ERR_INVALID;  // cannot hold in-flight items
+    // the ring must hold every item that can be in flight (depth iterations' worth)
+    if ((uint64_t)warps * c->batch * depth > next_pow2(cap)) return TQ_ERR_INVALID;
 
     tq_queue *q = nullptr;
     tq_status st = tq_create(cap, c->device, &q);
@@ -824,7 +839,12 @@ tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
     bp.timeout_ns = (unsigned long long)((c->timeout_s > 0 ? c->timeout_s : 60.0) * 1e9);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess) e = cudaEventRecord(e0, s);
-    if (e == cudaSuccess) e = launch_bench(c->variant, bp, blocks, block, s);
+    if (e == cudaSuccess) {
+        if (depth == 2)
+            e = launch_bench_pipe(cluster_v ? 2 : 1, csize, bp, blocks, block, s);
+        else
+            e = launch_bench(c->variant, bp, blocks, block, s);
+    }
     if (e == cudaSuccess) e = cudaEventRecord(e1, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(out_h, out, sizeof(out_h), cudaMemcpyDeviceToHost, s);
     unsigned status = 0;

@@ -5,6 +5,9 @@
 // (per-thread AFA, CAS-retry BASE, AN).  The retry ratio of
 // Fig 5 is atomics_issued / items.
 #include "internal.cuh"
+#ifdef TQ_DEBUG_PIPE
+#include <cstdio>
+#endif
 
 namespace tqk {
 
@@ -357,11 +360,265 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
     }
 }
 
+// ---------------------------------------------------------------------------
+// Pipelined variant (tq_bench_cfg.depth = 2): the group's proxy reserves the
+// Rear and Front tickets of iteration k+1 at the start of iteration k, so the
+// two atomics' latency overlaps the poll of iteration k, and the items of
+// iteration k+1 are published right after it; a dequeue then finds its item
+// already published one iteration earlier instead of waiting for another
+// group's producer to catch up.  Each warp still enqueues and dequeues b items
+// per iteration (<= 2b in flight).  Proxy group: GROUP 1 = CTA (thread 0,
+// bases through shared memory), 2 = thread-block cluster (CTA rank 0 thread 0,
+// bases written into every CTA's shared memory over DSMEM, one barrier.cluster
+// per iteration).  Not offered for single-warp groups: a group publishes
+// iteration k+1's items only after its poll of k, so a slow group delays its
+// consumers, and with 5920 independent warps the lag compounds until a
+// consumer holds a ticket a whole ring lap behind Rear (queue full at C = 2^20
+// with 0.4M items in flight, measured); CTA groups average it out.
+//
+// Deadlock freedom (all groups reserve the same gsz tickets on both counters
+// together, so ranges align): in a state where every group is blocked polling,
+// each group g has published all its Rear ranges but its last, and polls its
+// second-to-last Front range.  The globally last Rear range is unpublished but
+// no group polls the globally last Front range (it is some group's last), so
+// at most G-1 unpublished ranges can hold the G polled ranges: some group is
+// not blocked, and it publishes its last range before it polls again.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ unsigned cluster_ctarank()
+{
+    unsigned r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ unsigned cluster_nctarank()
+{
+    unsigned r;
+    asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r));
+    return r;
+}
+// store a u64 into CTA `rank`'s copy of the shared variable at `p`
+__device__ __forceinline__ void st_dsmem_u64(void *p, unsigned rank, unsigned long long v)
+{
+    const unsigned a = (unsigned)__cvta_generic_to_shared(p);
+    unsigned ra;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(rank));
+    asm volatile("st.shared::cluster.u64 [%0], %1;" ::"r"(ra), "l"(v) : "memory");
+}
+__device__ __forceinline__ void cluster_barrier()
+{
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <int GROUP>
+__global__ void __launch_bounds__(256) bench_pipe_kernel(const BenchParams p)
+{
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long warp_gid = ((unsigned long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const tq_device_view q = p.q;
+    const bool active = (int)lane < p.batch;
+    const unsigned wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+    unsigned n_enq = 0, n_deq = 0, atom = 0, empty = 0;
+    unsigned long long s_enq = 0, s_deq = 0, x_enq = 0, x_deq = 0, sink = 0;
+    const unsigned long long deadline = tq_globaltimer() + p.timeout_ns;
+    bool stop = false;
+
+    unsigned crank = 0, csize = 1;
+    if constexpr (GROUP == 2) {
+        crank = cluster_ctarank();
+        csize = cluster_nctarank();
+    }
+    // tickets per group per iteration and this lane's offset inside them
+    const unsigned long long gsz = (unsigned long long)nwb * csize * p.batch;
+    const unsigned long long off = ((unsigned long long)crank * nwb + wib) * p.batch + lane;
+    const bool leader = threadIdx.x == 0 && crank == 0;
+    // [parity][0 rear base, 1 front base, 2 stop]
+    __shared__ unsigned long long sb[2][3];
+
+    // Returns the group's (rear, front) bases reserved by the leader as
+    // (ra, fa); false if the group must stop.  One synchronisation.
+    auto distribute = [&](int par, unsigned long long ra, unsigned long long fa, unsigned long long lstop,
+                          unsigned long long *rb, unsigned long long *fb) -> bool {
+        if constexpr (GROUP == 1) {
+            if (leader) {
+                sb[par][0] = ra;
+                sb[par][1] = fa;
+            }
+            const bool st = __syncthreads_or(stop);
+            *rb = sb[par][0];
+            *fb = sb[par][1];
+            return !st;
+        } else {
+            if (leader) {
+                for (unsigned r = 0; r < csize; ++r) {
+                    st_dsmem_u64(&sb[par][0], r, ra);
+                    st_dsmem_u64(&sb[par][1], r, fa);
+                    st_dsmem_u64(&sb[par][2], r, lstop);
+                }
+            }
+            cluster_barrier();
+            *rb = sb[par][0];
+            *fb = sb[par][1];
+            return sb[par][2] == 0;
+        }
+    };
+    auto item_at = [&](int it) -> uint32_t {
+        return item_of(p.seed32, (warp_gid * (unsigned long long)p.iters + it) * p.batch + lane);
+    };
+    auto publish = [&](int it, unsigned long long rb) {
+        if (!active) return;
+        const unsigned long long et = rb + off;
+        const uint32_t item = item_at(it);
+        if (bench_publish(q, et, item)) {
+            ++n_enq;
+            const unsigned long long f = mix64(item);
+            s_enq += f;
+            x_enq ^= f;
+            if (p.enq_log) p.enq_log[et] = item;
+        } else {
+#ifdef TQ_DEBUG_PIPE
+            printf("full: warp %llu it %d ticket %llu slot %llx front %llu rear %llu\n", warp_gid, it, et,
+                   tq_ld_relaxed(q.slots + (et & q.mask)), tq_ld_relaxed(q.front), tq_ld_relaxed(q.rear));
+#endif
+            stop = true;
+        }
+    };
+
+    // prologue: reserve and publish iteration 0
+    unsigned long long ra = 0, fa = 0, rb = 0, fb = 0;
+    if (leader) {
+        ra = tq_atom_add(q.rear, gsz);
+        fa = tq_atom_add(q.front, gsz);
+        atom += 2;
+    }
+    bool go = distribute(0, ra, fa, 0ull, &rb, &fb);
+    if (go) publish(0, rb);
+    unsigned long long dt = fb + off;
+
+    for (int it = 0; go && it < p.iters; ++it) {
+        const bool more = it + 1 < p.iters;
+        unsigned long long lstop = 0;
+        if (more && leader) {  // iteration it+1's tickets, in flight during the poll
+            ra = tq_atom_add(q.rear, gsz);
+            fa = tq_atom_add(q.front, gsz);
+            atom += 2;
+            if constexpr (GROUP == 2) lstop = tq_status_read(q, (unsigned)warp_gid) != TQ_RUNNING;
+        }
+        if (active && !stop) {
+            uint32_t got_item = 0;
+            unsigned spins = 0;
+            bool have = false;
+            while (!have) {
+                have = tq_take(q, dt, &got_item);
+                if (!have) {
+                    ++empty;
+                    if ((++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {
+                        stop = true;
+                        break;
+                    }
+                }
+            }
+            if (have) {
+                ++n_deq;
+                const unsigned long long f = mix64(got_item);
+                s_deq += f;
+                x_deq ^= f;
+                if (p.deq_log) p.deq_log[dt] = got_item;
+                uint32_t x = got_item;
+                for (int w = 0; w < p.work_iters; ++w) x = x * 1664525u + 1013904223u;
+                sink += x;
+            }
+        }
+        if (!more) break;
+        go = distribute((it + 1) & 1, ra, fa, lstop, &rb, &fb);
+        if (go) publish(it + 1, rb);
+        dt = fb + off;
+    }
+
+    unsigned long long v[BO_COUNT_] = {n_enq, n_deq, atom, 0, empty, s_enq, s_deq, 0, 0, sink};
+#pragma unroll
+    for (int k = 0; k < BO_COUNT_; ++k) {
+        if (k == BO_XOR_ENQ || k == BO_XOR_DEQ) continue;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v[k] += __shfl_xor_sync(TQ_FULL_MASK, v[k], o);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        x_enq ^= __shfl_xor_sync(TQ_FULL_MASK, x_enq, o);
+        x_deq ^= __shfl_xor_sync(TQ_FULL_MASK, x_deq, o);
+    }
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < BO_COUNT_; ++k) {
+            if (k == BO_XOR_ENQ || k == BO_XOR_DEQ) continue;
+            if (v[k]) atomicAdd(p.out + k, v[k]);
+        }
+        atomicXor(p.out + BO_XOR_ENQ, x_enq);
+        atomicXor(p.out + BO_XOR_DEQ, x_deq);
+    }
+}
+
 template <int V>
 static cudaError_t launch_b(const BenchParams &p, int blocks, int block, cudaStream_t s)
 {
     bench_kernel<V><<<blocks, block, 0, s>>>(p);
     return cudaGetLastError();
+}
+
+// group: 0 warp, 1 CTA, 2 cluster of `cluster` CTAs (blocks % cluster == 0)
+cudaError_t launch_bench_pipe(int group, int cluster, const BenchParams &p, int blocks, int block,
+                              cudaStream_t s)
+{
+    if (group == 0) {
+        bench_pipe_kernel<0><<<blocks, block, 0, s>>>(p);
+    } else if (group == 1) {
+        bench_pipe_kernel<1><<<blocks, block, 0, s>>>(p);
+    } else {
+        if (cluster < 1 || blocks % cluster) return cudaErrorInvalidValue;
+        if (cluster > 8) {
+            cudaError_t e = cudaFuncSetAttribute(bench_pipe_kernel<2>,
+                                                 cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            if (e != cudaSuccess) return e;
+        }
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(blocks);
+        cfg.blockDim = dim3(block);
+        cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = cluster;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        return cudaLaunchKernelEx(&cfg, bench_pipe_kernel<2>, p);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t bench_pipe_occupancy(int block, int *blocks_per_sm)
+{
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, bench_pipe_kernel<1>, block, 0);
+}
+
+// co-resident clusters of `cluster` CTAs of `block` threads on this device
+cudaError_t bench_max_clusters(int cluster, int block, int *clusters)
+{
+    if (cluster > 8) {
+        cudaError_t e =
+            cudaFuncSetAttribute(bench_pipe_kernel<2>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (e != cudaSuccess) return e;
+    }
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(cluster * 148);
+    cfg.blockDim = dim3(block);
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = cluster;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaOccupancyMaxActiveClusters(clusters, bench_pipe_kernel<2>, &cfg);
 }
 
 cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int block, cudaStream_t s)

@@ -113,6 +113,10 @@ struct BenchParams {
 };
 cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int block, cudaStream_t s);
 cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm);
+cudaError_t launch_bench_pipe(int group, int cluster, const BenchParams &p, int blocks, int block,
+                              cudaStream_t s);
+cudaError_t bench_max_clusters(int cluster, int block, int *clusters);
+cudaError_t bench_pipe_occupancy(int block, int *blocks_per_sm);
 cudaError_t probe_ceiling(unsigned long long table_bytes, unsigned long long probes, int blocks_per_sm,
                           cudaStream_t s, double *g_per_s);
 
