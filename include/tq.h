@@ -310,6 +310,14 @@ const char *tq_strerror(tq_status s);
 tq_status tq_persistent_threads(int variant, int block, int device, int *threads_out);
 /* Library version string. */
 const char *tq_version(void);
+/* Device memory of queues and plans is drawn from a library-owned
+ * stream-ordered pool per device that keeps freed memory reserved, so a plan
+ * created right after another one of the same size (e.g. every step of a
+ * benchmark that rebuilds it from a host CSR) reuses it without cudaMalloc /
+ * cudaFree.  tq_memory_trim releases the cached, unused part of `device`'s
+ * pool to the driver (memory of live queues and plans stays).  Synchronises
+ * the device.  TQ_OK also when the pool was never created. */
+tq_status tq_memory_trim(int device);
 /* sizeof() of a public struct by name ("tq_csr", "bfs_opts", "bfs_stats",
  * "tq_device_view", "tq_counters", "tq_bench_cfg", "tq_bench_result"), 0 for
  * an unknown name: lets bindings check their struct mirrors without a GPU. */

@@ -95,6 +95,7 @@ EXPORTS = {
     "tq_persistent_threads": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                              ctypes.POINTER(ctypes.c_int)]),
     "tq_version": (ctypes.c_char_p, []),
+    "tq_memory_trim": (ctypes.c_int, [ctypes.c_int]),
     "tq_struct_size": (ctypes.c_size_t, [ctypes.c_char_p]),
     "tq_probe_ceiling": (ctypes.c_int, [ctypes.c_int, c_u64, c_u64, c_vp, ctypes.POINTER(c_dbl)]),
 }

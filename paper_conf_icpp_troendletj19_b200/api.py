@@ -359,5 +359,10 @@ def probe_ceiling(table_bytes: int, probes: int = 1 << 28, device: int = 0, stre
     return g.value
 
 
+def memory_trim(device: int = 0) -> None:
+    """`tq_memory_trim`: release the library pool's cached device memory."""
+    check(lib().tq_memory_trim(int(device)), "tq_memory_trim")
+
+
 def version() -> str:
     return lib().tq_version().decode()

@@ -10,11 +10,63 @@
 #include <stdlib.h>
 #include <string.h>
 
+#include <mutex>
 #include <new>
 
 #include "internal.cuh"
 
 using namespace tqk;
+
+namespace tqk {
+
+static cudaMemPool_t g_pools[256];
+static std::mutex g_pool_mu;
+
+static cudaMemPool_t lib_pool(int dev, bool create)
+{
+    std::lock_guard<std::mutex> lk(g_pool_mu);
+    if (dev < 0 || dev >= 256) return nullptr;
+    if (!g_pools[dev] && create) {
+        cudaMemPoolProps props{};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t pool = nullptr;
+        if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        unsigned long long keep = ~0ull;  // keep freed memory for the next plan
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+        g_pools[dev] = pool;
+    }
+    return g_pools[dev];
+}
+
+cudaError_t pool_alloc_raw(void **p, size_t bytes, cudaStream_t s)
+{
+    *p = nullptr;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    cudaMemPool_t pool = lib_pool(dev, true);
+    if (!pool) return cudaErrorMemoryAllocation;
+    e = cudaMallocFromPoolAsync(p, bytes > 0 ? bytes : 1, pool, s);
+    if (e == cudaErrorMemoryAllocation) {  // give cached blocks back, retry once
+        cudaGetLastError();
+        cudaStreamSynchronize(s);
+        cudaMemPoolTrimTo(pool, 0);
+        e = cudaMallocFromPoolAsync(p, bytes > 0 ? bytes : 1, pool, s);
+    }
+    return e;
+}
+
+void pool_free(void *p, cudaStream_t s)
+{
+    if (p) cudaFreeAsync(p, s);
+}
+
+}  // namespace tqk
 
 #define TQ_VERSION_STRING "tq-b200 0.1 (sm_100a)"
 
@@ -169,6 +221,17 @@ size_t tq_struct_size(const char *name)
     return 0;
 }
 
+tq_status tq_memory_trim(int device)
+{
+    DeviceGuard g(device);
+    if (!g.ok) return TQ_ERR_INVALID;
+    cudaMemPool_t pool = lib_pool(device, false);
+    if (!pool) return TQ_OK;
+    CK(cudaDeviceSynchronize());
+    CK(cudaMemPoolTrimTo(pool, 0));
+    return TQ_OK;
+}
+
 const char *tq_strerror(tq_status s)
 {
     switch (s) {
@@ -198,10 +261,12 @@ tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
     q->device = device;
     q->cap = next_pow2(capacity);
     while ((1ull << q->log2cap) < q->cap) ++q->log2cap;
-    cudaError_t e = cudaMalloc(&q->slots, q->cap * sizeof(unsigned long long));
-    if (e == cudaSuccess) e = cudaMalloc(&q->ctr, kCtrBytes);
+    cudaError_t e = pool_alloc(&q->slots, q->cap * sizeof(unsigned long long), 0);
+    if (e == cudaSuccess) e = pool_alloc(&q->ctr, kCtrBytes, 0);
     if (e != cudaSuccess) {
-        cudaFree(q->slots);
+        pool_free(q->slots, 0);
+        pool_free(q->ctr, 0);
+        cudaDeviceSynchronize();
         delete q;
         return from_cuda(e);
     }
@@ -226,8 +291,9 @@ tq_status tq_destroy(tq_queue *q)
 {
     if (!q) return TQ_OK;
     DeviceGuard g(q->device);
-    cudaFree(q->slots);
-    cudaFree(q->ctr);
+    // callers have finished with the queue (plans synchronise first)
+    pool_free(q->slots, 0);
+    pool_free(q->ctr, 0);
     delete q;
     return TQ_OK;
 }
@@ -289,22 +355,24 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     if (p->stream) cudaStreamSynchronize(p->stream);
     for (auto &e : p->ev)
         if (e) cudaEventDestroy(e);
-    if (p->owns_graph) {
-        cudaFree(p->row_ptr);
-        cudaFree(p->col);
-    }
-    cudaFree(p->W);
-    cudaFree(p->hub_base);
-    cudaFree(p->lvl8);
-    cudaFree(p->x8);
-    cudaFree(p->xd);
-    if (p->owns_wgt) cudaFree(p->wgt);
-    cudaFree(p->chunk_tab);
-    cudaFree(p->stats);
-    cudaFree(p->out_scratch);
     if (p->copy_stream) cudaStreamSynchronize(p->copy_stream);
+    // stream-ordered frees after everything that used the memory has finished
+    cudaStream_t fs = p->stream;
+    if (p->owns_graph) {
+        pool_free(p->row_ptr, fs);
+        pool_free(p->col, fs);
+    }
+    pool_free(p->W, fs);
+    pool_free(p->hub_base, fs);
+    pool_free(p->lvl8, fs);
+    pool_free(p->x8, fs);
+    pool_free(p->xd, fs);
+    if (p->owns_wgt) pool_free(p->wgt, fs);
+    pool_free(p->chunk_tab, fs);
+    pool_free(p->stats, fs);
+    pool_free(p->out_scratch, fs);
     for (int b = 0; b < 2; ++b) {
-        cudaFree(p->dbuf[b]);
+        pool_free(p->dbuf[b], fs);
         if (p->bfs_done[b]) cudaEventDestroy(p->bfs_done[b]);
         if (p->copy_done[b]) cudaEventDestroy(p->copy_done[b]);
     }
@@ -378,8 +446,8 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         p->col = const_cast<int32_t *>(gph->col);
     } else {
         p->owns_graph = true;
-        e = cudaMalloc(&p->row_ptr, (size_t)(n + 1) * sizeof(int64_t));
-        if (e == cudaSuccess) e = cudaMalloc(&p->col, (size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t));
+        e = pool_alloc(&p->row_ptr, (size_t)(n + 1) * sizeof(int64_t), p->stream);
+        if (e == cudaSuccess) e = pool_alloc(&p->col, (size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t), p->stream);
         if (e == cudaSuccess)
             e = cudaMemcpyAsync(p->row_ptr, gph->row_ptr, (size_t)(n + 1) * sizeof(int64_t),
                                 cudaMemcpyHostToDevice, p->stream);
@@ -393,22 +461,22 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
             p->wgt = const_cast<int32_t *>(weights);
         } else {
             p->owns_wgt = true;
-            e = cudaMalloc(&p->wgt, (size_t)nnz * sizeof(int32_t));
+            e = pool_alloc(&p->wgt, (size_t)nnz * sizeof(int32_t), p->stream);
             if (e == cudaSuccess)
                 e = cudaMemcpyAsync(p->wgt, weights, (size_t)nnz * sizeof(int32_t), cudaMemcpyHostToDevice,
                                     p->stream);
             if (e != cudaSuccess) return fail(from_cuda(e));
         }
     }
-    e = cudaMalloc(&p->W, (size_t)n * sizeof(unsigned long long));
-    if (e == cudaSuccess) e = cudaMalloc(&p->hub_base, (size_t)n * sizeof(int32_t));
+    e = pool_alloc(&p->W, (size_t)n * sizeof(unsigned long long), p->stream);
+    if (e == cudaSuccess) e = pool_alloc(&p->hub_base, (size_t)n * sizeof(int32_t), p->stream);
     if (task == kTaskBFS) {
-        if (e == cudaSuccess) e = cudaMalloc(&p->lvl8, (size_t)n);
-        if (e == cudaSuccess) e = cudaMalloc(&p->x8, (size_t)n);
+        if (e == cudaSuccess) e = pool_alloc(&p->lvl8, (size_t)n, p->stream);
+        if (e == cudaSuccess) e = pool_alloc(&p->x8, (size_t)n, p->stream);
     } else {
-        if (e == cudaSuccess) e = cudaMalloc(&p->xd, (size_t)n * sizeof(unsigned));
+        if (e == cudaSuccess) e = pool_alloc(&p->xd, (size_t)n * sizeof(unsigned), p->stream);
     }
-    if (e == cudaSuccess) e = cudaMalloc(&p->stats, kStatCount * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = pool_alloc(&p->stats, kStatCount * sizeof(unsigned long long), p->stream);
     if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMallocHost(&p->ctr_h, 8 * sizeof(unsigned long long));
     for (auto &ev : p->ev)
@@ -641,7 +709,7 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
     if (host_l || host_p) {
         // two device output pairs + a copy stream, allocated on first use
         if (!p->dbuf[0]) {
-            for (int b = 0; b < 2; ++b) CK(cudaMalloc(&p->dbuf[b], 2 * vb));
+            for (int b = 0; b < 2; ++b) CK(pool_alloc(&p->dbuf[b], 2 * vb, p->stream));
             CK(cudaStreamCreateWithFlags(&p->copy_stream, cudaStreamNonBlocking));
             for (int b = 0; b < 2; ++b) {
                 CK(cudaEventCreateWithFlags(&p->bfs_done[b], cudaEventDisableTiming));
@@ -703,7 +771,7 @@ tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *p
         const tq_status st = plan_launch(p, root, level_out, parent_out);
         return st == TQ_OK ? plan_finish(p, stats) : st;
     }
-    if (!p->out_scratch) CK(cudaMalloc(&p->out_scratch, (size_t)p->n * 2 * sizeof(int32_t)));
+    if (!p->out_scratch) CK(pool_alloc(&p->out_scratch, (size_t)p->n * 2 * sizeof(int32_t), p->stream));
     int32_t *dl = level_out ? (host_l ? p->out_scratch : level_out) : nullptr;
     int32_t *dp = parent_out ? (host_p ? p->out_scratch + p->n : parent_out) : nullptr;
     tq_status st = plan_launch(p, root, dl, dp);

@@ -1170,11 +1170,11 @@ cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int3
     int32_t *nch = nullptr;
     void *tmp = nullptr;
     size_t tmp_bytes = 0;
-    cudaError_t e = cudaMalloc(&nch, (size_t)n * sizeof(int32_t));
+    cudaError_t e = pool_alloc(&nch, (size_t)n * sizeof(int32_t), s);
     if (e != cudaSuccess) return e;
     count_chunks_kernel<<<grid_for(n, 256), 256, 0, s>>>(row_ptr, n, chunk, nch);
     e = cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, nch, hub_base, (int)n, s);
-    if (e == cudaSuccess) e = cudaMalloc(&tmp, tmp_bytes);
+    if (e == cudaSuccess) e = pool_alloc(&tmp, tmp_bytes, s);
     if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, nch, hub_base, (int)n, s);
     int32_t last_base = 0, last_n = 0;
     if (e == cudaSuccess)
@@ -1185,7 +1185,7 @@ cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int3
     const int64_t total = (int64_t)last_base + last_n;
     if (e == cudaSuccess && total > 0) {
         int2 *tab = nullptr;
-        e = cudaMalloc(&tab, (size_t)total * sizeof(int2));
+        e = pool_alloc(&tab, (size_t)total * sizeof(int2), s);
         if (e == cudaSuccess) {
             fill_chunks_kernel<<<grid_for(n, 256), 256, 0, s>>>(row_ptr, n, chunk, hub_base, tab);
             e = cudaGetLastError();
@@ -1194,12 +1194,12 @@ cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int3
                 *chunk_tab_out = tab;
                 *n_chunks_out = total;
             } else {
-                cudaFree(tab);
+                pool_free(tab, s);
             }
         }
     }
-    cudaFree(tmp);
-    cudaFree(nch);
+    pool_free(tmp, s);
+    pool_free(nch, s);
     return e;
 }
 

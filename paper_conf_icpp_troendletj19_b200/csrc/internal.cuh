@@ -29,6 +29,19 @@ __device__ __forceinline__ unsigned long long *per_lane_addr(unsigned long long 
     return p + (tq_lane() & zero);
 }
 
+// Device memory of queues and plans comes from a library-owned, stream-ordered
+// pool (one per device) that keeps freed memory reserved (release threshold =
+// max), so plans created and destroyed every step -- bench.py's e2e leg builds
+// one from the host CSR per step -- do not pay cudaMalloc / cudaFree of
+// multi-GB buffers each time.  tq_memory_trim() returns it to the driver.
+cudaError_t pool_alloc_raw(void **p, size_t bytes, cudaStream_t s);
+void pool_free(void *p, cudaStream_t s);
+template <typename T>
+inline cudaError_t pool_alloc(T **p, size_t bytes, cudaStream_t s)
+{
+    return pool_alloc_raw(reinterpret_cast<void **>(p), bytes, s);
+}
+
 #ifdef TQ_AB_PROF
 constexpr int kStatCount = 24;  // 16..19: idle / prolog / expand / enqueue SM cycles (A/B builds only)
 #else

@@ -358,3 +358,20 @@ def test_ring_wraps_within_runs(tq):
 def test_probe_ceiling_measures(tq):
     g = tq.probe_ceiling(1 << 24, 1 << 22)
     assert 1.0 < g < 10000.0
+
+
+def test_plans_recycled_through_the_memory_pool(tq):
+    """Plans built from host CSRs of different sizes, destroyed and rebuilt
+    (their device memory recycled by the library's stream-ordered pool), and
+    the pool trimmed in between: every run stays identical to the oracle."""
+    graphs = [kronecker_csr(12, 16, 3), grid_csr(64, 64), kronecker_csr(12, 16, 3), kronecker_csr(11, 8, 4)]
+    for i, g in enumerate(graphs):
+        root = int(sample_roots(g.row_ptr, 1, seed=i)[0])
+        lv = np.empty(g.n_vertices, dtype=np.int32)
+        pa = np.empty(g.n_vertices, dtype=np.int32)
+        with tq.BfsPlan(g.row_ptr, g.col, parents="min_id") as plan:
+            st = plan.run(root, lv, pa)
+        check_against_oracle(g, root, lv, pa, st, min_id=True)
+        if i == 1:
+            tq.memory_trim(0)
+    tq.memory_trim(0)
