@@ -166,12 +166,21 @@ def main():
         run_reference(args, kind, a, ef, n_roots)
         return
 
+    # TQ_DIST_BACKEND=gloo (test only): several ranks sharing the visible
+    # GPUs (device = LOCAL_RANK mod count) with host-side collectives, to
+    # exercise the N > 1 path on a one-GPU box; the product path is NCCL
+    backend = os.environ.get("TQ_DIST_BACKEND", "nccl")
+    local = local % max(torch.cuda.device_count(), 1) if backend == "gloo" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    coll_dev = dev if backend == "nccl" else None  # device of the collectives' tensors
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
 
     import paper_conf_icpp_troendletj19_b200 as tq
     from paper_conf_icpp_troendletj19_b200 import multiroot
@@ -216,7 +225,7 @@ def main():
     regrows = plan.regrows
 
     # NCCL all-gather of per-rank stats (the only collective; outside the data path)
-    agg = multiroot.aggregate(multiroot.gather(multiroot.local_vector(all_stats, ms_total), dist, dev))
+    agg = multiroot.aggregate(multiroot.gather(multiroot.local_vector(all_stats, ms_total), dist, coll_dev))
     ms_max = agg["ms"]
     te_all = agg["traversed_edges"]
     reached_all = agg["reached"]
@@ -278,9 +287,9 @@ def main():
             step_s.append([round(ts1 - ts0, 3), round(ts2 - ts1, 3), round(time.perf_counter() - ts2, 3)])
         torch.cuda.synchronize(dev)
         sec = time.perf_counter() - t0
-        secv = torch.tensor([sec, te_e2e], dtype=torch.float64, device=dev)
+        secv = torch.tensor([sec, te_e2e], dtype=torch.float64, device=coll_dev)
         if dist:
-            o2 = torch.empty(world * 2, dtype=torch.float64, device=dev)
+            o2 = torch.empty(world * 2, dtype=torch.float64, device=coll_dev)
             dist.all_gather_into_tensor(o2, secv)
             o2 = o2.view(world, 2).cpu().numpy()
             sec_max, te_tot = float(o2[:, 0].max()), float(o2[:, 1].sum())
@@ -379,11 +388,14 @@ def run_reference(args, kind, a, ef, n_roots):
     v = te / sec / 1e9
     print(json.dumps({
         "impl": "reference", "metric": "BFS GTEPS (batched multi-root, persistent-thread RF/AN queue)",
-        "value": round(v, 6), "unit": "GTEPS", "n_gpus": 1, "steps": args.steps,
+        "value": round(v, 6), "unit": "GTEPS", "n_gpus": int(os.environ.get("WORLD_SIZE", 1)),
+        "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(sec / args.steps * 1e3, 3),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
         "dtype": "int32/int64 (integer path)", "data": "synthetic",
-        "config": {"workload": args.workload},
+        "config": {"workload": args.workload, "graph": f"{kind} {a}" + (f" ef{ef}" if ef else ""),
+                   "n_vertices": int(rp.size - 1), "nnz": int(cl.size), "roots_total": len(roots),
+                   "parallelism": "rank 0 only: the sequential oracle on one host core"},
         "cpu_baseline": {"value": round(v, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",
                          "sample": f"one root of the workload per step ({args.steps} steps)"},
         "e2e": {"value": round(v, 6), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
