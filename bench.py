@@ -147,6 +147,7 @@ def main():
     ap.add_argument("--variant", default="rf_an")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-queue", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=20.0)
     ap.add_argument("--parents", default="any", choices=["any", "min_id"])
     args = ap.parse_args()
@@ -255,6 +256,29 @@ def main():
                               "32 B L2 sector each: the level-mirror probe) vs tq_probe_ceiling over a "
                               "table of the mirror's size, measured in this run"}
 
+    # ---- queue throughput on this GPU (BASELINE metric's second half, config 2
+    # at full occupancy; outside the BFS timed region, device-timed by tq_bench) ----
+    queue = None
+    if not args.no_queue:
+        from inputs import fingerprint, item_of
+        queue = {"unit": "M ops/s (enqueue + dequeue)", "items": 1 << 24, "per_gpu": True,
+                 "capacity": 1 << 22, "runs": []}
+        for v, b, d in (("rf_an", 1, 1), ("rf_an", 32, 1), ("rf_an_cta", 32, 2), ("per_thread_afa", 32, 1),
+                        ("atomic_ceiling", 32, 1)):
+            r = tq.queue_bench(v, warps=0, batch=b, items=1 << 24, capacity=1 << 22, seed=3, depth=d,
+                               device=local, timeout_s=30)
+            rec = {"variant": v, "batch": b, "depth": d, "threads": 32 * r["warps"],
+                   "mops": round(2 * r["items"] / (r["ms"] * 1e-3) / 1e6, 1),
+                   "atomics_per_item": round(r["atomics"] / r["items"], 4)}
+            if v == "atomic_ceiling":
+                rec = {"variant": v, "threads": rec["threads"],
+                       "same_address_atomics_per_s_G": round(r["atomics"] / (r["ms"] * 1e-3) / 1e9, 3)}
+            else:
+                exp = fingerprint(item_of(3, np.arange(r["items"])))
+                rec["conserved"] = ((r["enq"], r["sum_enq"], r["xor_enq"]) == tuple(exp) and
+                                    (r["deq"], r["sum_deq"], r["xor_deq"]) == tuple(exp))
+            queue["runs"].append(rec)
+
     # ---- e2e through the public API with host buffers (pinned), every step ----
     e2e = None
     if not args.no_e2e:
@@ -342,6 +366,7 @@ def main():
                          "alg_bytes_per_launch": int(alg_bytes),
                          "avg_launch_ms": round(avg_kernel_s * 1e3, 4)},
             "roofline_l2_probe": probe_roof,
+            "queue": queue,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,
