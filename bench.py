@@ -208,7 +208,8 @@ def main():
     # the expansion's second ceiling, measured live on this GPU (outside the
     # timed region): random 1-byte L2 probes over a table the size of the
     # level mirror, at the persistent kernel's shape
-    probe_g = tq.probe_ceiling(max(n, 1 << 12), 1 << 28, device=local) if kind == "kron" else None
+    mirror_bytes = n if n <= (1 << 25) else (n + 7) // 8 * 4  # byte / nibble mirror (R8)
+    probe_g = tq.probe_ceiling(max(mirror_bytes, 1 << 12), 1 << 28, device=local) if kind == "kron" else None
 
     # ---- timed region: K steps, barrier + sync on both sides, device events ----
     if dist:

@@ -174,7 +174,9 @@ struct bfs_plan {
     bool owns_graph = false;
     unsigned long long *W = nullptr;
     int32_t *hub_base = nullptr;
-    uint8_t *lvl8 = nullptr;
+    unsigned *mir = nullptr;                  // level mirror (bytes or nibbles)
+    int mirror_bits = 8;
+    size_t mirror_bytes = 0;
     uint8_t *x8 = nullptr;
     unsigned *xd = nullptr;                   // SSSP: expanded-distance marker
     int32_t *wgt = nullptr;                   // SSSP: edge weights (device)
@@ -193,7 +195,7 @@ struct bfs_plan {
     int32_t *dbuf[2] = {nullptr, nullptr};    // batch: double-buffered device outputs
     cudaStream_t copy_stream = nullptr;       // batch: D2H copies
     cudaEvent_t bfs_done[2] = {nullptr, nullptr}, copy_done[2] = {nullptr, nullptr};
-    size_t l2_window = 0;                     // persisting-L2 window over lvl8
+    size_t l2_window = 0;                     // persisting-L2 window over the level mirror
     size_t l2_limit_saved = 0;                // device persisting-L2 limit to restore
     bool l2_limit_set = false;
     unsigned long long next_ticket = 0;
@@ -364,7 +366,7 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     }
     pool_free(p->W, fs);
     pool_free(p->hub_base, fs);
-    pool_free(p->lvl8, fs);
+    pool_free(p->mir, fs);
     pool_free(p->x8, fs);
     pool_free(p->xd, fs);
     if (p->owns_wgt) pool_free(p->wgt, fs);
@@ -471,7 +473,15 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     e = pool_alloc(&p->W, (size_t)n * sizeof(unsigned long long), p->stream);
     if (e == cudaSuccess) e = pool_alloc(&p->hub_base, (size_t)n * sizeof(int32_t), p->stream);
     if (task == kTaskBFS) {
-        if (e == cudaSuccess) e = pool_alloc(&p->lvl8, (size_t)n, p->stream);
+        // Level mirror width (R8): a nibble per vertex when a byte
+        // mirror would exceed 32 MB (it then no longer stays L2-resident next
+        // to the col stream; measured: s26 -3.6%, s24 / grid +2-4% with
+        // nibbles), RF/AN only.  TQ_MIRROR_BITS=4|8 overrides (experiments).
+        p->mirror_bits = (o.variant == TQ_VARIANT_RF_AN && n > (1ll << 25)) ? 4 : 8;
+        const char *mb = getenv("TQ_MIRROR_BITS");
+        if (mb && o.variant == TQ_VARIANT_RF_AN && (mb[0] == '4' || mb[0] == '8')) p->mirror_bits = mb[0] - '0';
+        p->mirror_bytes = p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 7) / 8 * 4;
+        if (e == cudaSuccess) e = pool_alloc(&p->mir, p->mirror_bytes, p->stream);
         if (e == cudaSuccess) e = pool_alloc(&p->x8, (size_t)n, p->stream);
     } else {
         if (e == cudaSuccess) e = pool_alloc(&p->xd, (size_t)n * sizeof(unsigned), p->stream);
@@ -523,7 +533,7 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         int max_win = 0, max_persist = 0;
         cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, gdev);
         cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, gdev);
-        size_t w = (size_t)n;
+        size_t w = p->mirror_bytes;
         if (w > (size_t)max_win) w = (size_t)max_win;
         if (w > (size_t)max_persist) w = (size_t)max_persist;
         size_t cur = 0;
@@ -582,7 +592,8 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.W = p->W;
     bp.chunk_tab = p->chunk_tab;
     bp.hub_base = p->hub_base;
-    bp.lvl8 = p->lvl8;
+    bp.mir = p->mir;
+    bp.mirror_bits = p->mirror_bits;
     bp.x8 = p->x8;
     bp.xd = p->xd;
     bp.wgt = p->wgt;

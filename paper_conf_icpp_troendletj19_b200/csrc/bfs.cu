@@ -51,7 +51,18 @@ constexpr int kU = TQ_AB_KU;         // 32-edge rounds in flight per lane
 // spills; interleaved A/B on B200 (results/ab_occupancy_r01.md): 5 blocks
 // beat 6 by 1-3% on Kronecker and 8% on the grid, 4 and 8 blocks are slower.
 constexpr int kMinBlocks = TQ_AB_MINB;
-constexpr unsigned kLvlSat = 254;    // byte mirror: 0..253 exact, 254 = ">= 254", 255 = unreached
+constexpr unsigned kLvlSat = 254;    // byte: 0..253 exact, 254 = ">= 254", 255 = unreached / none
+// Level mirror (R8), MIR bits per vertex:
+//   MIR = 8: one byte per vertex: 0..253 exact-or-stale-high, 254 = ">= 254",
+//            255 = unreached; updated with a plain store.
+//   MIR = 4: one nibble per vertex, eight per 32-bit word (u in word u >> 3,
+//            bits 4 * (u & 7)): 0..13, 14 = ">= 14", 15 = unreached; updated
+//            with a CAS loop.  Half the bytes, so it stays L2-resident where a
+//            byte mirror does not (scale 26: 34 MB vs 67 MB); the plan picks it
+//            when the byte mirror would exceed 32 MB.
+template <int MIR> struct Mirror;
+template <> struct Mirror<8> { static constexpr unsigned kSat = 254; };
+template <> struct Mirror<4> { static constexpr unsigned kSat = 14; };
 // bound on CAS retries of one operation; reaching it can only mean a broken
 // queue state (the loops are lock-free), which is reported as a timeout
 constexpr unsigned kMaxEnqRetries = 1u << 24;
@@ -91,6 +102,12 @@ __device__ __forceinline__ int64_t ld_nc_i64(const int64_t *p)
     return v;
 }
 
+__device__ __forceinline__ unsigned ld_cg_u32(const unsigned *p, unsigned long long pol)
+{
+    unsigned v;
+    asm volatile("ld.global.cg.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
 __device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long long pol)
 {
     unsigned v;
@@ -413,9 +430,10 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
 // ---------------------------------------------------------------------------
 // The persistent kernel
 // ---------------------------------------------------------------------------
-template <int VARIANT, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks>
+template <int VARIANT, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, int MIR = 8>
 __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsParams p)
 {
+    constexpr unsigned kMirSat = Mirror<MIR>::kSat;
     __shared__ uint32_t stage_all[kWarps][kStageCap];
     const unsigned lane = threadIdx.x & 31;
     const unsigned warp_gid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -752,29 +770,33 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 #pragma unroll
                 for (int j = 0; j < KU; ++j) cand[j] = val[j] && off[j] < w[j];
             } else {
-                // prefilter 1: the byte level mirror (L2-resident; stale values
-                // are never below the true level, R8)
-                unsigned m8[KU];
+                // prefilter 1: the level mirror (L2-resident; stale values are
+                // never below the true level, R8)
+                unsigned b8[KU];  // the probed mirror byte / word
 #pragma unroll
                 for (int j = 0; j < KU; ++j) {
-                    // offers at level >= 254 cannot be filtered by the saturated
-                    // mirror: skip the probe (saves a dependent round trip on deep
-                    // graphs, e.g. the grid's 8,191 levels) and go to atomicMin
-                    const bool deep = lv1[j] >= kLvlSat;
-                    m8[j] = (val[j] && !deep) ? ld_cg_u8(p.lvl8 + u[j], pol_keep) : kLvlSat;
+                    // offers at a level >= the mirror's saturation cannot be
+                    // filtered: skip the probe (saves a dependent round trip on
+                    // deep graphs, e.g. the grid's 8,191 levels), go to atomicMin
+                    const bool deep = lv1[j] >= kMirSat;
+                    if constexpr (MIR == 8)
+                        b8[j] = (val[j] && !deep) ? ld_cg_u8((const uint8_t *)p.mir + u[j], pol_keep) : 0xFFu;
+                    else
+                        b8[j] = (val[j] && !deep) ? ld_cg_u32(p.mir + ((unsigned)u[j] >> 3), pol_keep) : ~0u;
                 }
 #ifdef TQ_AB_PROF
                 long long tc;  // after the mirror probes returned
-                asm volatile("mov.u64 %0, %%clock64;" : "=l"(tc) : "r"(m8[0]), "r"(m8[KU - 1]), "r"(m8[1]), "r"(m8[2]));
+                asm volatile("mov.u64 %0, %%clock64;" : "=l"(tc) : "r"(b8[0]), "r"(b8[KU - 1]), "r"(b8[1]), "r"(b8[2]));
                 TQ_PROF_ADD(5, tc - tb);
 #endif
                 bool tie[KU];
                 bool any_tie = false;
 #pragma unroll
                 for (int j = 0; j < KU; ++j) {
-                    const bool known = m8[j] < kLvlSat;  // exact-or-stale-high level
-                    tie[j] = val[j] && min_id && known && m8[j] == lv1[j];
-                    cand[j] = val[j] && !(known && m8[j] <= lv1[j]);
+                    const unsigned m8 = MIR == 8 ? b8[j] : (b8[j] >> (((unsigned)u[j] & 7u) << 2)) & 0xFu;
+                    const bool known = m8 < kMirSat;  // exact-or-stale-high level
+                    tie[j] = val[j] && min_id && known && m8 == lv1[j];
+                    cand[j] = val[j] && !(known && m8 <= lv1[j]);
                     any_tie |= tie[j];
                 }
                 // prefilter 2 (min-id parents only): the packed word, only for
@@ -825,7 +847,23 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         const unsigned L1 = (unsigned)(co >> 32);
                         const unsigned oldhi = c ? (unsigned)(atomicMin(p.W + cv, co) >> 32) : 0u;
                         const bool nt = c && oldhi > L1;  // level strictly lowered: (re)discovered
-                        if (nt) st_u8(p.lvl8 + cv, L1 < kLvlSat ? L1 : kLvlSat);
+                        // Lower v's mirror entry.  It only ever receives levels
+                        // installed by a successful atomicMin (>= the final
+                        // level): the mirror stays stale-high, the only
+                        // property the prefilter needs.  Byte: a plain store;
+                        // nibble: a CAS loop on its word.
+                        if constexpr (MIR == 8) {
+                            if (nt) st_u8((uint8_t *)p.mir + cv, L1 < kMirSat ? L1 : kMirSat);
+                        } else if (nt && L1 < kMirSat) {
+                            unsigned *wp = p.mir + (cv >> 3);
+                            const unsigned sh = (cv & 7u) << 2;
+                            unsigned old = tq_ld_relaxed_u32(wp);
+                            while (((old >> sh) & 0xFu) > L1) {
+                                const unsigned got = atomicCAS(wp, old, (old & ~(0xFu << sh)) | (L1 << sh));
+                                if (got == old) break;
+                                old = got;
+                            }
+                        }
                         n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, nt && oldhi != 0xffffffffu));
                         const unsigned m = __ballot_sync(TQ_FULL_MASK, nt);
                         if (nt) stage[wr + __popc(m & tq_lanemask_lt())] = cv;
@@ -850,7 +888,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         const unsigned L1 = (unsigned)(off[j] >> 32);
                         if ((old >> 32) > L1) {  // level strictly lowered: (re)discovered
                             nt[j] = true;
-                            if constexpr (TASK == kTaskBFS) st_u8(p.lvl8 + u[j], L1 < kLvlSat ? L1 : kLvlSat);
                             re = (old >> 32) != 0xffffffffull;
                         }
                     }
@@ -954,7 +991,11 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
         p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
-        if (p.lvl8) p.lvl8[i] = (i == root) ? 0 : 255;
+        if (p.mir && p.mirror_bits == 8) {
+            ((uint8_t *)p.mir)[i] = (i == root) ? 0 : 255;
+        } else if (p.mir && i < (n + 7) / 8) {  // nibbles: 15 = unreached, root's = 0
+            p.mir[i] = (i == (root >> 3)) ? ~(0xFu << ((root & 7) << 2)) : ~0u;
+        }
         if (p.x8) p.x8[i] = 255;
         if (p.xd) p.xd[i] = 0xffffffffu;
     }
@@ -1101,7 +1142,7 @@ cudaError_t launch_queue_reset(const tq_device_view &q, cudaStream_t s)
     return cudaGetLastError();
 }
 
-template <int V, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks>
+template <int V, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, int MIR = 8>
 static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStream_t s)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
@@ -1111,11 +1152,11 @@ static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStrea
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
     if (p.l2_window_bytes) {
-        // keep the byte level mirror (probed once per edge) resident in the
+        // keep the level mirror (probed once per edge) resident in the
         // persisting part of L2 while the col stream and the per-task arrays
         // pass through
         attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-        attr[0].val.accessPolicyWindow.base_ptr = (void *)p.lvl8;
+        attr[0].val.accessPolicyWindow.base_ptr = (void *)p.mir;
         attr[0].val.accessPolicyWindow.num_bytes = p.l2_window_bytes;
         attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
         attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
@@ -1123,7 +1164,7 @@ static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStrea
         cfg.attrs = attr;
         cfg.numAttrs = 1;
     }
-    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, TASK, KU, MINB>, p);
+    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, TASK, KU, MINB, MIR>, p);
 }
 
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
@@ -1134,7 +1175,9 @@ cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, i
         return launch_v<TQ_VARIANT_RF_AN, kTaskSSSP>(p, blocks, block, s);
     }
     switch (variant) {
-    case TQ_VARIANT_RF_AN: return launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
+    case TQ_VARIANT_RF_AN:
+        if (p.mirror_bits == 4) return launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 4>(p, blocks, block, s);
+        return launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
     case TQ_VARIANT_PER_THREAD_AFA: return launch_v<TQ_VARIANT_PER_THREAD_AFA>(p, blocks, block, s);
     case TQ_VARIANT_CAS_RETRY: return launch_v<TQ_VARIANT_CAS_RETRY>(p, blocks, block, s);
     case TQ_VARIANT_AN: return launch_v<TQ_VARIANT_AN>(p, blocks, block, s);

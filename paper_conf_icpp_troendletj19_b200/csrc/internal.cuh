@@ -80,7 +80,8 @@ struct BfsParams {
     unsigned long long *W;     // packed (level << 32) | parent, ~0 = unreached
     const int2 *chunk_tab;     // chunk id -> {vertex, k}
     const int32_t *hub_base;   // vertex -> first chunk id (read for hubs only)
-    uint8_t *lvl8;             // byte level mirror (prefilter), 255 = unreached
+    unsigned *mir;             // level mirror (prefilter): bytes or nibbles, see bfs.cu Mirror<>
+    int mirror_bits;           // 8 (byte per vertex) or 4 (nibble; RF/AN BFS on large graphs)
     uint8_t *x8;               // level at which the vertex was expanded (saturating byte)
     unsigned *xd;              // SSSP: distance at which the vertex was expanded
     const int32_t *wgt;        // SSSP: edge weights (one per CSR entry), else null
@@ -92,7 +93,7 @@ struct BfsParams {
     int backoff_ns;            // max idle back-off, 0 = none
     int parent_rule;           // TQ_PARENT_ANY / TQ_PARENT_MIN_ID (include/tq.h)
     unsigned long long timeout_ns;
-    size_t l2_window_bytes;    // persisting-L2 window over lvl8 (0 = none)
+    size_t l2_window_bytes;    // persisting-L2 window over the level mirror (0 = none)
     unsigned delay_ns;         // test only: schedule perturbation (bfs_opts.debug_delay_ns)
     unsigned delay_seed;
     // first-lap bounds: tickets below these are known empty at run start

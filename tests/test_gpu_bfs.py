@@ -375,3 +375,29 @@ def test_plans_recycled_through_the_memory_pool(tq):
         if i == 1:
             tq.memory_trim(0)
     tq.memory_trim(0)
+
+
+@pytest.mark.parametrize("bits", ["4", "8"])
+@pytest.mark.parametrize("parents", ["any", "min_id"])
+def test_level_mirror_widths(tq, monkeypatch, bits, parents):
+    """Both level-mirror widths (R8; the plan picks nibbles above
+    2^25 vertices, TQ_MIRROR_BITS forces one): identical levels on graphs
+    whose depth stays below, crosses and far exceeds the nibble's saturation
+    (14) and the byte's (254), with delay injection perturbing the schedule."""
+    monkeypatch.setenv("TQ_MIRROR_BITS", bits)
+    graphs = [kronecker_csr(12, 16, 5), grid_csr(40, 23),
+              edges_to_csr(np.arange(599), np.arange(1, 600), 600, "path600"), tree4_csr(20000)]
+    for g in graphs:
+        rp, col = to_dev(g)
+        roots = [0, int(sample_roots(g.row_ptr, 1, seed=9)[0])]
+        with tq.BfsPlan(rp, col, parents=parents, timeout_s=20) as plan:
+            import torch
+            lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+            pa = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+            for root in roots:
+                st = plan.run(root, lv, pa)
+                check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
+        with tq.BfsPlan(rp, col, parents=parents, timeout_s=20, debug_delay_ns=2000,
+                        debug_delay_seed=3) as plan:
+            st = plan.run(roots[1], lv, pa)
+            check_against_oracle(g, roots[1], lv, pa, st, min_id=parents == "min_id")
