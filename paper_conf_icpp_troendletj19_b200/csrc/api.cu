@@ -482,7 +482,9 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         if (mb && o.variant == TQ_VARIANT_RF_AN && (mb[0] == '4' || mb[0] == '8')) p->mirror_bits = mb[0] - '0';
         p->mirror_bytes = p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 7) / 8 * 4;
         if (e == cudaSuccess) e = pool_alloc(&p->mir, p->mirror_bytes, p->stream);
-        if (e == cudaSuccess) e = pool_alloc(&p->x8, (size_t)n, p->stream);
+        // expanded-level markers: same width as the mirror
+        if (e == cudaSuccess)
+            e = pool_alloc(&p->x8, p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 1) / 2, p->stream);
     } else {
         if (e == cudaSuccess) e = pool_alloc(&p->xd, (size_t)n * sizeof(unsigned), p->stream);
     }

@@ -683,16 +683,33 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             if (!(item & CHUNK_FLAG)) {
                 // expanded-level marker (R7): a vertex already
                 // expanded at a level <= L has offered <= L+1 to every
-                // neighbour, so this token has nothing left to do.  A byte,
-                // saturating like the mirror (254 = "expanded at >= 254",
-                // which never skips).
-                const unsigned xprev = ld_relaxed_u8(p.x8 + v);
-                if (xprev < kLvlSat && xprev <= L) {
-                    skipped = true;
-                    hi = lo;
-                    nch = 0;
+                // neighbour, so this token has nothing left to do.  Same
+                // width as the mirror, saturating like it ("expanded at >=
+                // sat" never skips).  The nibble form rewrites the byte it
+                // read: a concurrent update of the pair vertex can be undone,
+                // which only restores an older (higher) marker -- a weaker
+                // skip, never a wrong one (a vertex's expansion levels only
+                // fall).
+                if constexpr (MIR == 8) {
+                    const unsigned xprev = ld_relaxed_u8(p.x8 + v);
+                    if (xprev < kLvlSat && xprev <= L) {
+                        skipped = true;
+                        hi = lo;
+                        nch = 0;
+                    } else {
+                        st_u8(p.x8 + v, L < kLvlSat ? L : kLvlSat);
+                    }
                 } else {
-                    st_u8(p.x8 + v, L < kLvlSat ? L : kLvlSat);
+                    const unsigned xb = ld_relaxed_u8(p.x8 + ((unsigned)v >> 1));
+                    const unsigned sh = ((unsigned)v & 1u) << 2;
+                    const unsigned xprev = (xb >> sh) & 0xFu;
+                    if (xprev < kMirSat && xprev <= L) {
+                        skipped = true;
+                        hi = lo;
+                        nch = 0;
+                    } else if (L < kMirSat) {
+                        st_u8(p.x8 + ((unsigned)v >> 1), (xb & ~(0xFu << sh)) | (L << sh));
+                    }
                 }
             }
             }
@@ -996,7 +1013,7 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
         } else if (p.mir && i < (n + 7) / 8) {  // nibbles: 15 = unreached, root's = 0
             p.mir[i] = (i == (root >> 3)) ? ~(0xFu << ((root & 7) << 2)) : ~0u;
         }
-        if (p.x8) p.x8[i] = 255;
+        if (p.x8 && (p.mirror_bits == 8 || i < (n + 1) / 2)) p.x8[i] = 255;  // byte / nibble markers
         if (p.xd) p.xd[i] = 0xffffffffu;
     }
     if (blockIdx.x == 0) {
