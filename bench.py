@@ -341,6 +341,7 @@ def main():
                "sample": f"{len(done)} of the {len(roots)} roots of the same graph, sequential "
                          f"BFS levels only ({sec:.1f} s of CPU)"}
 
+    csr_mb = ((n + 1) * 8 + col.numel() * 4) / 1e6
     if rank == 0:
         line = {
             "metric": "BFS GTEPS (batched multi-root, persistent-thread RF/AN queue)",
@@ -359,7 +360,9 @@ def main():
                        "n_vertices": n, "nnz": int(col.numel()), "roots_total": len(roots),
                        "roots_per_rank": len(mine), "variant": args.variant,
                        "parallelism": f"roots split over {world} rank(s), graph replicated",
-                       "l2": "inputs larger than L2 (CSR >> 126 MB)",
+                       "l2": ("inputs larger than L2 (CSR %.0f MB > 126 MB)" % csr_mb) if csr_mb > 126 else
+                             ("inputs smaller than L2 (CSR %.1f MB; not flushed between roots: a parity-size "
+                              "workload, not the metric's)" % csr_mb),
                        "persistent_threads": all_stats[0]["persistent_threads"]},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak,
                          "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": traffic,
