@@ -564,13 +564,11 @@ static cudaError_t launch_b(const BenchParams &p, int blocks, int block, cudaStr
     return cudaGetLastError();
 }
 
-// group: 0 warp, 1 CTA, 2 cluster of `cluster` CTAs (blocks % cluster == 0)
+// group: 1 CTA, 2 cluster of `cluster` CTAs (blocks % cluster == 0)
 cudaError_t launch_bench_pipe(int group, int cluster, const BenchParams &p, int blocks, int block,
                               cudaStream_t s)
 {
-    if (group == 0) {
-        bench_pipe_kernel<0><<<blocks, block, 0, s>>>(p);
-    } else if (group == 1) {
+    if (group == 1) {
         bench_pipe_kernel<1><<<blocks, block, 0, s>>>(p);
     } else {
         if (cluster < 1 || blocks % cluster) return cudaErrorInvalidValue;

@@ -40,7 +40,9 @@ for b in [int(x) for x in args.batches.split(",")]:
             print(json.dumps({"v": v, "depth": d, "cluster": c, "b": b, "error": str(e)}), flush=True)
             continue
         g = {"rf_an": 1, "rf_an_cta": 8, "rf_an_cluster": 8 * max(c, 1)}[v]
-        ws = sorted({w for w in (1, 8, 64, 128, 512, 1024, 2048, 4096) if w % g == 0 and w <= full} | {full})
+        # a CTA group may be a single warp (1-warp blocks): its own linear baseline
+        ws = sorted({w for w in (1, 8, 64, 128, 512, 1024, 2048, 4096)
+                     if (w % g == 0 or (v == "rf_an_cta" and w == 1)) and w <= full} | {full})
         base = None
         for w in ws:
             try:
