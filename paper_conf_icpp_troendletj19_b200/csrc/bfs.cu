@@ -441,6 +441,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     // owner lanes of one round's atomicMin candidates (ids go to the stage tail)
     __shared__ uint8_t cown_all[kWarps][32 * KU];
     uint8_t *cown = cown_all[threadIdx.x >> 5];
+    // nibble mirror: their probed mirror words (the CAS's expected value)
+    __shared__ unsigned cw_all[MIR == 4 ? kWarps : 1][MIR == 4 ? 32 * KU : 1];
+    unsigned *cw = cw_all[MIR == 4 ? (threadIdx.x >> 5) : 0];
     const tq_device_view q = p.q;
     const unsigned long long cap = q.mask + 1;
     const int chunk = p.chunk;
@@ -777,6 +780,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             TQ_PROF_ADD(4, tb - ta);
 #endif
             bool cand[KU];
+            unsigned b8[KU];  // BFS: the probed mirror byte / word
             if constexpr (TASK == kTaskSSSP) {
                 // prefilter: the packed word itself (dist, parent) -- stale
                 // values are never below the true word, so skipping offers
@@ -789,7 +793,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             } else {
                 // prefilter 1: the level mirror (L2-resident; stale values are
                 // never below the true level, R8)
-                unsigned b8[KU];  // the probed mirror byte / word
 #pragma unroll
                 for (int j = 0; j < KU; ++j) {
                     // offers at a level >= the mirror's saturation cannot be
@@ -849,6 +852,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         const unsigned k = ncand + __popc(m & tq_lanemask_lt());
                         stage[cnt + k] = (uint32_t)u[j];
                         cown[k] = (uint8_t)(ownp >> (8 * j));
+                        if constexpr (MIR == 4) cw[k] = b8[j];
                     }
                     ncand += __popc(m);
                 }
@@ -860,26 +864,29 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         const bool c = i < ncand;
                         const uint32_t cv = c ? stage[cnt + i] : 0u;
                         const unsigned long long co = tq_shfl64(offer, c ? cown[i] : 0u);
+                        const unsigned cb = (MIR == 4 && c) ? cw[i] : ~0u;
                         __syncwarp();  // all reads of this slice before the in-place writes
                         const unsigned L1 = (unsigned)(co >> 32);
                         const unsigned oldhi = c ? (unsigned)(atomicMin(p.W + cv, co) >> 32) : 0u;
                         const bool nt = c && oldhi > L1;  // level strictly lowered: (re)discovered
                         // Lower v's mirror entry.  It only ever receives levels
-                        // installed by a successful atomicMin (>= the final
-                        // level): the mirror stays stale-high, the only
-                        // property the prefilter needs.  Byte: a plain store;
-                        // nibble: a CAS loop on its word.
+                        // v has held (installed by a successful atomicMin, so
+                        // >= the final level): the mirror stays stale-high,
+                        // the only property the prefilter needs.  Byte: a
+                        // plain store.  Nibble: one fire-and-forget CAS from
+                        // the word probed this round (no wait; if another of
+                        // the word's 8 vertices changed meanwhile it fails and
+                        // v's nibble stays high), and a failed candidate whose
+                        // probe read a nibble above v's current level repairs
+                        // it the same way, so a missed lowering costs one
+                        // extra atomicMin, not one per later probe.
                         if constexpr (MIR == 8) {
                             if (nt) st_u8((uint8_t *)p.mir + cv, L1 < kMirSat ? L1 : kMirSat);
-                        } else if (nt && L1 < kMirSat) {
-                            unsigned *wp = p.mir + (cv >> 3);
+                        } else {
+                            const unsigned nv = nt ? L1 : oldhi;  // v's level now
                             const unsigned sh = (cv & 7u) << 2;
-                            unsigned old = tq_ld_relaxed_u32(wp);
-                            while (((old >> sh) & 0xFu) > L1) {
-                                const unsigned got = atomicCAS(wp, old, (old & ~(0xFu << sh)) | (L1 << sh));
-                                if (got == old) break;
-                                old = got;
-                            }
+                            if (c && nv < kMirSat && nv < ((cb >> sh) & 0xFu))
+                                atomicCAS(p.mir + (cv >> 3), cb, (cb & ~(0xFu << sh)) | (nv << sh));
                         }
                         n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, nt && oldhi != 0xffffffffu));
                         const unsigned m = __ballot_sync(TQ_FULL_MASK, nt);
