@@ -257,29 +257,6 @@ def main():
                               "32 B L2 sector each: the level-mirror probe) vs tq_probe_ceiling over a "
                               "table of the mirror's size, measured in this run"}
 
-    # ---- queue throughput on this GPU (BASELINE metric's second half, config 2
-    # at full occupancy; outside the BFS timed region, device-timed by tq_bench) ----
-    queue = None
-    if not args.no_queue:
-        from inputs import fingerprint, item_of
-        queue = {"unit": "M ops/s (enqueue + dequeue)", "items": 1 << 24, "per_gpu": True,
-                 "capacity": 1 << 22, "runs": []}
-        for v, b, d in (("rf_an", 1, 1), ("rf_an", 32, 1), ("rf_an_cta", 32, 2), ("per_thread_afa", 32, 1),
-                        ("atomic_ceiling", 32, 1)):
-            r = tq.queue_bench(v, warps=0, batch=b, items=1 << 24, capacity=1 << 22, seed=3, depth=d,
-                               device=local, timeout_s=30)
-            rec = {"variant": v, "batch": b, "depth": d, "threads": 32 * r["warps"],
-                   "mops": round(2 * r["items"] / (r["ms"] * 1e-3) / 1e6, 1),
-                   "atomics_per_item": round(r["atomics"] / r["items"], 4)}
-            if v == "atomic_ceiling":
-                rec = {"variant": v, "threads": rec["threads"],
-                       "same_address_atomics_per_s_G": round(r["atomics"] / (r["ms"] * 1e-3) / 1e9, 3)}
-            else:
-                exp = fingerprint(item_of(3, np.arange(r["items"])))
-                rec["conserved"] = ((r["enq"], r["sum_enq"], r["xor_enq"]) == tuple(exp) and
-                                    (r["deq"], r["sum_deq"], r["xor_deq"]) == tuple(exp))
-            queue["runs"].append(rec)
-
     # ---- e2e through the public API with host buffers (pinned), every step ----
     e2e = None
     if not args.no_e2e:
@@ -326,6 +303,30 @@ def main():
                "step_s_create_batch_destroy": step_s,
                "timed": "host perf_counter per step around bfs_plan_create(pinned host CSR: H2D) + "
                         "bfs_plan_run_batch(all roots, pinned host level/parent: D2H per root), synchronised"}
+
+    # ---- queue throughput on this GPU (BASELINE metric's second half, config 2
+    # at full occupancy; outside the BFS timed region, device-timed by tq_bench;
+    # after the e2e leg, whose first plan would otherwise grow the memory pool) ----
+    queue = None
+    if not args.no_queue:
+        from inputs import fingerprint, item_of
+        queue = {"unit": "M ops/s (enqueue + dequeue)", "items": 1 << 24, "per_gpu": True,
+                 "capacity": 1 << 22, "runs": []}
+        for v, b, d in (("rf_an", 1, 1), ("rf_an", 32, 1), ("rf_an_cta", 32, 2), ("per_thread_afa", 32, 1),
+                        ("atomic_ceiling", 32, 1)):
+            r = tq.queue_bench(v, warps=0, batch=b, items=1 << 24, capacity=1 << 22, seed=3, depth=d,
+                               device=local, timeout_s=30)
+            rec = {"variant": v, "batch": b, "depth": d, "threads": 32 * r["warps"],
+                   "mops": round(2 * r["items"] / (r["ms"] * 1e-3) / 1e6, 1),
+                   "atomics_per_item": round(r["atomics"] / r["items"], 4)}
+            if v == "atomic_ceiling":
+                rec = {"variant": v, "threads": rec["threads"],
+                       "same_address_atomics_per_s_G": round(r["atomics"] / (r["ms"] * 1e-3) / 1e9, 3)}
+            else:
+                exp = fingerprint(item_of(3, np.arange(r["items"])))
+                rec["conserved"] = ((r["enq"], r["sum_enq"], r["xor_enq"]) == tuple(exp) and
+                                    (r["deq"], r["sum_deq"], r["xor_deq"]) == tuple(exp))
+            queue["runs"].append(rec)
 
     # ---- CPU baseline: the oracle, 1 core, bounded sample, rank 0 at N=1 ----
     cpu = None
