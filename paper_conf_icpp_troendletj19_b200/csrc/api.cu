@@ -176,6 +176,7 @@ struct bfs_plan {
     int32_t *hub_base = nullptr;
     unsigned *mir = nullptr;                  // level mirror (bytes or nibbles)
     int mirror_bits = 8;
+    bool auto_blocks = false;                 // threads == 0: full grid, one block per SM on deep graphs
     size_t mirror_bytes = 0;
     uint8_t *x8 = nullptr;
     unsigned *xd = nullptr;                   // SSSP: expanded-distance marker
@@ -524,6 +525,7 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         p->blocks = (o.threads + p->block - 1) / p->block;
     } else {
         p->blocks = full;
+        p->auto_blocks = task == kTaskBFS && !getenv("TQ_NO_DEEP_GRID");
     }
     if (p->blocks < 1) p->blocks = 1;
     const char *l2env = getenv("TQ_L2_WINDOW");  // "0": experiments only
@@ -684,6 +686,15 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
                 (double)h[16], (double)h[17], (double)h[18], (double)h[19], (double)h[20], (double)h[21],
                 (double)(h[18] - h[20] - h[21] - h[22]), (double)h[22]);
 #endif
+    }
+    // Deep graphs: a BFS of >= 1,024 levels runs a few thousand
+    // vertices per level at a time; a full persistent grid then spends L2 on
+    // idle polls of its 189K held tickets (the paper's too-many-threads
+    // dilemma).  After such a run the plan (same graph) launches one
+    // block per SM: grid 4096^2 53 -> ~46 ms.  Only when threads == 0.
+    if (p->auto_blocks && status == TQ_FINISHED && p->stats_h[ST_MAX_LEVEL] >= 1024) {
+        const int deep_blocks = sm_count(p->device);
+        if (p->blocks > deep_blocks) p->blocks = deep_blocks;
     }
     if (status == TQ_FINISHED) return TQ_OK;
     if (status == TQ_ABORTED_FULL) return TQ_ERR_QUEUE_FULL;

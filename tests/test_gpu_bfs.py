@@ -401,3 +401,31 @@ def test_level_mirror_widths(tq, monkeypatch, bits, parents):
                         debug_delay_seed=3) as plan:
             st = plan.run(roots[1], lv, pa)
             check_against_oracle(g, roots[1], lv, pa, st, min_id=parents == "min_id")
+
+
+def test_deep_graph_plans_shrink_the_grid(tq):
+    """threads == 0: after a run of >= 1,024 levels the plan launches one
+    block per SM; shallow graphs keep the full grid; an
+    explicit thread count is never changed.  Results stay exact."""
+    import torch
+    full = tq.persistent_threads()
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    deep = edges_to_csr(np.arange(2999), np.arange(1, 3000), 3000, "path3000")
+    rp, col = to_dev(deep)
+    lv = torch.empty(deep.n_vertices, dtype=torch.int32, device="cuda")
+    pa = torch.empty_like(lv)
+    with tq.BfsPlan(rp, col, timeout_s=30) as plan:
+        st1 = plan.run(0, lv, pa)
+        check_against_oracle(deep, 0, lv, pa, st1)
+        st2 = plan.run(1500, lv, pa)
+        check_against_oracle(deep, 1500, lv, pa, st2)
+    assert st1["persistent_threads"] == full and st2["persistent_threads"] == sms * 256
+    with tq.BfsPlan(rp, col, threads=4096, timeout_s=30) as plan:
+        plan.run(0, lv, pa)
+        assert plan.run(7, lv, pa)["persistent_threads"] == 4096
+    g = kronecker_csr(12, 16, 5)
+    rp, col = to_dev(g)
+    lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+    with tq.BfsPlan(rp, col) as plan:
+        plan.run(int(sample_roots(g.row_ptr, 1, 1)[0]), lv, None)
+        assert plan.run(int(sample_roots(g.row_ptr, 1, 2)[0]), lv, None)["persistent_threads"] == full
