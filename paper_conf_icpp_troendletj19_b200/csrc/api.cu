@@ -9,6 +9,7 @@
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
+#include <time.h>
 
 #include <mutex>
 #include <new>
@@ -64,6 +65,39 @@ cudaError_t pool_alloc_raw(void **p, size_t bytes, cudaStream_t s)
 void pool_free(void *p, cudaStream_t s)
 {
     if (p) cudaFreeAsync(p, s);
+}
+
+// Small pinned host buffers (a plan's statistics / counter read-back) are
+// recycled through a free list: cudaFreeHost can wait for the whole device,
+// which made plan teardown take up to 0.5 s in the e2e leg.
+static std::mutex g_pin_mu;
+static void *g_pin_free[64];
+static int g_pin_n = 0;
+static constexpr size_t kPinBytes = 256;  // >= kStatCount and 8 counters of 8 bytes
+
+static cudaError_t pinned_small_alloc(void **p)
+{
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        if (g_pin_n > 0) {
+            *p = g_pin_free[--g_pin_n];
+            return cudaSuccess;
+        }
+    }
+    return cudaMallocHost(p, kPinBytes);
+}
+
+static void pinned_small_free(void *p)
+{
+    if (!p) return;
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        if (g_pin_n < 64) {
+            g_pin_free[g_pin_n++] = p;
+            return;
+        }
+    }
+    cudaFreeHost(p);
 }
 
 }  // namespace tqk
@@ -355,10 +389,22 @@ tq_status bfs_plan_destroy(bfs_plan *p)
 {
     if (!p) return TQ_OK;
     DeviceGuard g(p->device);
+    // TQ_DEBUG_DESTROY=1: per-step timing to stderr (diagnostics only)
+    const bool dbg = getenv("TQ_DEBUG_DESTROY") != nullptr;
+    double tt[8] = {0};
+    int ti = 0;
+    auto tick = [&]() {
+        if (!dbg) return;
+        timespec ts;
+        clock_gettime(CLOCK_MONOTONIC, &ts);
+        tt[ti++] = ts.tv_sec + ts.tv_nsec * 1e-9;
+    };
+    tick();
     if (p->stream) cudaStreamSynchronize(p->stream);
     for (auto &e : p->ev)
         if (e) cudaEventDestroy(e);
     if (p->copy_stream) cudaStreamSynchronize(p->copy_stream);
+    tick();
     // stream-ordered frees after everything that used the memory has finished
     cudaStream_t fs = p->stream;
     if (p->owns_graph) {
@@ -379,13 +425,21 @@ tq_status bfs_plan_destroy(bfs_plan *p)
         if (p->bfs_done[b]) cudaEventDestroy(p->bfs_done[b]);
         if (p->copy_done[b]) cudaEventDestroy(p->copy_done[b]);
     }
+    tick();
     if (p->copy_stream) cudaStreamDestroy(p->copy_stream);
-    if (p->stats_h) cudaFreeHost(p->stats_h);
-    if (p->ctr_h) cudaFreeHost(p->ctr_h);
+    pinned_small_free(p->stats_h);
+    pinned_small_free(p->ctr_h);
+    tick();
     if (p->l2_window) cudaCtxResetPersistingL2Cache();
+    tick();
     if (p->l2_limit_set) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, p->l2_limit_saved);
+    tick();
     tq_destroy(p->q);
     tq_destroy(p->q1);
+    tick();
+    if (dbg)
+        fprintf(stderr, "TQDESTROY sync %.4f frees %.4f host %.4f l2reset %.4f l2limit %.4f queues %.4f\n",
+                tt[1] - tt[0], tt[2] - tt[1], tt[3] - tt[2], tt[4] - tt[3], tt[5] - tt[4], tt[6] - tt[5]);
     delete p;
     return TQ_OK;
 }
@@ -490,8 +544,9 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         if (e == cudaSuccess) e = pool_alloc(&p->xd, (size_t)n * sizeof(unsigned), p->stream);
     }
     if (e == cudaSuccess) e = pool_alloc(&p->stats, kStatCount * sizeof(unsigned long long), p->stream);
-    if (e == cudaSuccess) e = cudaMallocHost(&p->stats_h, kStatCount * sizeof(unsigned long long));
-    if (e == cudaSuccess) e = cudaMallocHost(&p->ctr_h, 8 * sizeof(unsigned long long));
+    static_assert(kStatCount * sizeof(unsigned long long) <= kPinBytes, "pinned block too small");
+    if (e == cudaSuccess) e = pinned_small_alloc(reinterpret_cast<void **>(&p->stats_h));
+    if (e == cudaSuccess) e = pinned_small_alloc(reinterpret_cast<void **>(&p->ctr_h));
     for (auto &ev : p->ev)
         if (e == cudaSuccess) e = cudaEventCreate(&ev);
     if (e != cudaSuccess) return fail(from_cuda(e));
