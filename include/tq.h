@@ -140,7 +140,11 @@ typedef struct {
 typedef struct {
     uint64_t capacity;  /* queue slots; 0 = 2^ceil(log2(2V)), at least 2^16   */
     int threads;        /* persistent threads; 0 = SMs x occupancy (P:63,
-                           P:83 "just enough threads to saturate")           */
+                           P:83 "just enough threads to saturate"), and a
+                           BFS plan whose run reached >= 1,024 levels uses
+                           one block per SM for its later runs (deep graphs:
+                           the too-many-threads side of the dilemma);
+                           > 0 = exactly this many (rounded up to blocks)    */
     int block;          /* threads per block; 0 = 256                        */
     int chunk;          /* sub-task size: max edges per task token (P:153
                            "a fixed number of uniformly complex sub-tasks";
