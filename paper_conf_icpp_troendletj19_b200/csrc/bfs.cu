@@ -1052,7 +1052,49 @@ __global__ void __launch_bounds__(256) bfs_unpack_kernel(const BfsParams p, int3
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     unsigned long long reached = 0, degsum = 0;
     unsigned maxl = 0;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    // 4 vertices per thread with 16-byte accesses when every array is 16-byte
+    // aligned (HBM-bound: W 8 B + row_ptr 8 B read, level + parent 8 B written
+    // per vertex); the scalar loop takes the tail and unaligned outputs
+    const bool vec = ((reinterpret_cast<uintptr_t>(p.W) | reinterpret_cast<uintptr_t>(p.row_ptr) |
+                       reinterpret_cast<uintptr_t>(level) | reinterpret_cast<uintptr_t>(parent)) & 15) == 0;
+    int64_t done = 0;
+    if (vec) {
+        const int64_t n4 = n / 4;
+        for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n4; k += stride) {
+            const int64_t i = 4 * k;
+            const ulonglong2 w01 = *reinterpret_cast<const ulonglong2 *>(p.W + i);
+            const ulonglong2 w23 = *reinterpret_cast<const ulonglong2 *>(p.W + i + 2);
+            const unsigned long long w[4] = {w01.x, w01.y, w23.x, w23.y};
+            int4 lv, pa;
+            int *lvp = &lv.x, *pap = &pa.x;
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const unsigned l = (unsigned)(w[j] >> 32);
+                const bool r = l != 0xffffffffu;
+                lvp[j] = r ? (int32_t)l : -1;
+                pap[j] = r ? (int32_t)(uint32_t)w[j] : -1;
+                if (r) {
+                    ++reached;
+                    maxl = max(maxl, l);
+                }
+                any |= r;
+            }
+            if (level) *reinterpret_cast<int4 *>(level + i) = lv;
+            if (parent) *reinterpret_cast<int4 *>(parent + i) = pa;
+            if (any) {
+                const longlong2 r01 = *reinterpret_cast<const longlong2 *>(p.row_ptr + i);
+                const longlong2 r23 = *reinterpret_cast<const longlong2 *>(p.row_ptr + i + 2);
+                const long long r4 = ld_nc_i64(p.row_ptr + i + 4);
+                const long long rp[5] = {r01.x, r01.y, r23.x, r23.y, r4};
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    if (lvp[j] >= 0) degsum += (unsigned long long)(rp[j + 1] - rp[j]);
+            }
+        }
+        done = 4 * n4;
+    }
+    for (int64_t i = done + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
         const unsigned long long w = p.W[i];
         const unsigned l = (unsigned)(w >> 32);
         const bool r = l != 0xffffffffu;
