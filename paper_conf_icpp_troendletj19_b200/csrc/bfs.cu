@@ -1008,21 +1008,53 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 // a2: state + queue init for one run.  W[:] = unreached, W[root] = (0, root);
 // the root is published at ticket t0 (Front = Done = t0, Rear = t0 + 1).
 // ---------------------------------------------------------------------------
+// Fill nbytes of a 16-byte-aligned buffer with 0xFF, byte `sb` ANDed with
+// `smask` (the root's mirror entry), 16 bytes per store.
+__device__ __forceinline__ void fill_ff(uint8_t *buf, int64_t nbytes, int64_t sb, unsigned smask,
+                                        int64_t tid, int64_t stride)
+{
+    const int64_t n16 = nbytes / 16;
+    for (int64_t c = tid; c < n16; c += stride) {
+        uint4 v = make_uint4(~0u, ~0u, ~0u, ~0u);
+        if (sb >= 16 * c && sb < 16 * c + 16) {
+            unsigned *w = &v.x;
+            const int b = (int)(sb - 16 * c);
+            w[b >> 2] &= ~((~smask & 0xFFu) << (8 * (b & 3)));
+        }
+        reinterpret_cast<uint4 *>(buf)[c] = v;
+    }
+    for (int64_t b = 16 * n16 + tid; b < nbytes; b += stride) buf[b] = (uint8_t)(b == sb ? (0xFFu & smask) : 0xFFu);
+}
+
 __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long long t0,
                                 unsigned long long t1)
 {
     const int64_t n = p.n_vertices;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-        p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
-        if (p.mir && p.mirror_bits == 8) {
-            ((uint8_t *)p.mir)[i] = (i == root) ? 0 : 255;
-        } else if (p.mir && i < (n + 7) / 8) {  // nibbles: 15 = unreached, root's = 0
-            p.mir[i] = (i == (root >> 3)) ? ~(0xFu << ((root & 7) << 2)) : ~0u;
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    // W: 4 entries (32 bytes) per store pair; plan buffers are pool
+    // allocations (256-byte aligned)
+    const int64_t n4 = n / 4;
+    for (int64_t k = tid; k < n4; k += stride) {
+        ulonglong2 a = make_ulonglong2(~0ull, ~0ull), b = a;
+        const int64_t i = 4 * k;
+        if (root >= i && root < i + 4) {
+            unsigned long long *e = root < i + 2 ? &a.x : &b.x;
+            e[(root - i) & 1] = (unsigned long long)(uint32_t)root;
         }
-        if (p.x8 && (p.mirror_bits == 8 || i < (n + 1) / 2)) p.x8[i] = 255;  // byte / nibble markers
-        if (p.xd) p.xd[i] = 0xffffffffu;
+        reinterpret_cast<ulonglong2 *>(p.W + i)[0] = a;
+        reinterpret_cast<ulonglong2 *>(p.W + i)[1] = b;
     }
+    for (int64_t i = 4 * n4 + tid; i < n; i += stride)
+        p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
+    if (p.mir) {  // level mirror: bytes (root's = 0) or nibbles (15 = unreached, root's = 0)
+        if (p.mirror_bits == 8)
+            fill_ff((uint8_t *)p.mir, n, root, 0x00u, tid, stride);
+        else
+            fill_ff((uint8_t *)p.mir, (n + 7) / 8 * 4, root >> 1, ~(0xFu << ((root & 1) << 2)), tid, stride);
+    }
+    if (p.x8) fill_ff(p.x8, p.mirror_bits == 8 ? n : (n + 1) / 2, -1, 0xFFu, tid, stride);  // markers
+    if (p.xd) fill_ff(reinterpret_cast<uint8_t *>(p.xd), 4 * n, -1, 0xFFu, tid, stride);
     if (blockIdx.x == 0) {
         if (threadIdx.x < TQ_STATUS_COPIES) p.q.status[threadIdx.x * TQ_STATUS_STRIDE] = TQ_RUNNING;
         if (threadIdx.x < kStatCount) p.stats[threadIdx.x] = 0;
