@@ -35,7 +35,20 @@ constexpr int kWarps = kBlock / 32;
 #ifndef TQ_AB_STAGE
 #define TQ_AB_STAGE 512
 #endif
-constexpr int kStageCap = TQ_AB_STAGE;  // staged tokens per warp (2 KiB smem)
+#ifndef TQ_AB_STAGE_BYTE
+#define TQ_AB_STAGE_BYTE 768
+#endif
+// Staged tokens per warp (2-3 KiB smem). A larger stage publishes children in
+// bigger, later batches: fewer label-correcting re-scans, less work visible to
+// idle warps. Measured (results/ab_occupancy_r01.md, stage sweeps): 768 is best
+// for byte-mirror graphs (<= 2^25 vertices; kron24 3.87 -> 3.62 ms), 512 for
+// nibble-mirror ones (kron26 16.02 vs 16.27 ms).
+// SSSP keeps 512 (its re-enqueues are label-correcting by design; 768 measured
+// 103 vs 117 G edges/s at s24).
+template <int MIR, int TASK> __host__ __device__ constexpr int stage_cap()
+{
+    return (MIR == 8 && TASK == kTaskBFS) ? TQ_AB_STAGE_BYTE : TQ_AB_STAGE;
+}
 // A/B builds (scripts/ab_bfs.py) override these with -D; the defaults are
 // the measured best.
 #ifndef TQ_AB_KU
@@ -434,6 +447,7 @@ template <int VARIANT, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, 
 __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsParams p)
 {
     constexpr unsigned kMirSat = Mirror<MIR>::kSat;
+    constexpr int kStageCap = stage_cap<MIR, TASK>();
     __shared__ uint32_t stage_all[kWarps][kStageCap];
     const unsigned lane = threadIdx.x & 31;
     const unsigned warp_gid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
