@@ -43,8 +43,8 @@ constexpr int kWarps = kBlock / 32;
 // idle warps. Measured (results/ab_occupancy_r01.md, stage sweeps): 768 is best
 // for byte-mirror graphs (<= 2^25 vertices; kron24 3.87 -> 3.62 ms), 512 for
 // nibble-mirror ones (kron26 16.02 vs 16.27 ms).
-// SSSP keeps 512 (its re-enqueues are label-correcting by design; 768 measured
-// 103 vs 117 G edges/s at s24).
+// SSSP keeps 512, the setting it was tuned and validated with (its run-to-run
+// spread, 18.6-25.4 ms per s24 source at either size, hides any difference).
 template <int MIR, int TASK> __host__ __device__ constexpr int stage_cap()
 {
     return (MIR == 8 && TASK == kTaskBFS) ? TQ_AB_STAGE_BYTE : TQ_AB_STAGE;
