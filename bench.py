@@ -96,6 +96,17 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(s)}
 
 
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def make_graph(kind, a, ef, device):
     import inputs.gpu as gg
     gg.build()
@@ -225,6 +236,12 @@ def main():
         dist.barrier()
     ms_total = e0.elapsed_time(e1)
     regrows = plan.regrows
+    # outputs of the last timed root, from the long-running plan that was timed
+    # (its tickets have crossed the 2^32 wrap of the sequence tags many times)
+    last_root = mine[-1] if mine else None
+    last_level = level.cpu().numpy() if mine else None
+    last_parent = parent.cpu().numpy() if mine else None
+    plan_tickets = plan.tickets()
 
     # NCCL all-gather of per-rank stats (the only collective; outside the data path)
     agg = multiroot.aggregate(multiroot.gather(multiroot.local_vector(all_stats, ms_total), dist, coll_dev))
@@ -337,14 +354,20 @@ def main():
     # ---- CPU baseline: the oracle, 1 core, bounded sample, rank 0 at N=1 ----
     cpu = None
     parity = None
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and not args.no_cpu and last_root is not None:
+        import oracle
         col_host = col.cpu().numpy()
-        teps, done, sec, lv0 = cpu_oracle_sample(rp_host, col_host, mine, args.cpu_budget)
-        plan2 = tq.BfsPlan(row_ptr, col, variant=args.variant, device=local, parents=args.parents)
-        plan2.run(done[0], level, parent)
-        parity = bool(np.array_equal(level.cpu().numpy(), lv0))
-        plan2.close()
+        # the oracle's first root is the last timed root: its levels are the
+        # parity reference for the timed plan's output (and part of the sample)
+        sample_roots_ = [last_root] + [r for r in mine if r != last_root]
+        teps, done, sec, lv0 = cpu_oracle_sample(rp_host, col_host, sample_roots_, args.cpu_budget)
+        rule, bad = oracle.validate_tree(rp_host, col_host, last_root, last_level, last_parent)
+        parity = {"root": int(last_root), "levels_identical": bool(np.array_equal(last_level, lv0)),
+                  "parents_graph500_valid": rule == 0, "validate_rule": rule,
+                  "plan_tickets_after_timed_runs": [int(t) for t in plan_tickets],
+                  "what": "last timed root of the timed (long-running) plan vs the oracle"}
         cpu = {"value": teps / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+               "nproc": os.cpu_count(), "cpu_model": cpu_model(),
                "sample": f"{len(done)} of the {len(roots)} roots of the same graph, sequential "
                          f"BFS levels only ({sec:.1f} s of CPU)"}
 
@@ -370,7 +393,8 @@ def main():
                        "l2": ("inputs larger than L2 (CSR %.0f MB > 126 MB)" % csr_mb) if csr_mb > 126 else
                              ("inputs smaller than L2 (CSR %.1f MB; not flushed between roots: a parity-size "
                               "workload, not the metric's)" % csr_mb),
-                       "persistent_threads": all_stats[0]["persistent_threads"]},
+                       "persistent_threads": max((st["persistent_threads"] for st in all_stats),
+                                                 default=tq.persistent_threads(args.variant, device=local))},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak,
                          "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": traffic,
                          "kernel": "bfs_persistent_kernel<RF_AN>", "peak_source": peak_src,
@@ -382,7 +406,7 @@ def main():
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk.summary(),
-            "parity_sampled_root_levels_identical": parity,
+            "parity": parity,
             "graph_gen_s": round(t_gen, 2),
             "queue_regrows": regrows,
         }

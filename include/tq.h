@@ -94,6 +94,13 @@ tq_status tq_destroy(tq_queue *q);
  * timeout, which can leave slots written but untaken. */
 tq_status tq_reset(tq_queue *q, void *stream);
 
+/* Reset to the empty state with the counters at ticket t0 instead of 0:
+ * Front = Rear = Done = t0, and every slot holds "empty" for the unique
+ * ticket t in [t0, t0 + C) that maps to it (seq == (uint32)t).  Lets a test
+ * start a queue just below a 2^32 boundary of the 32-bit sequence tags.
+ * t0 < 2^63; stream-ordered like tq_reset. */
+tq_status tq_reset_at(tq_queue *q, uint64_t t0, void *stream);
+
 /* Queue status words (replicated; see tq_device.cuh). */
 enum { TQ_RUNNING = 0, TQ_FINISHED = 1, TQ_ABORTED_FULL = 2, TQ_ABORTED_TIMEOUT = 3 };
 
@@ -174,6 +181,18 @@ typedef struct {
                            == 1, so tokens are expanded late and with stale
                            levels.  0 = off (default); at most 1,000,000     */
     uint32_t debug_delay_seed;
+    int mirror_bits;    /* level-mirror width (R8): 0 = auto (a nibble
+                           per vertex when a byte mirror would exceed 32 MB,
+                           RF_AN only; else a byte), 8 = byte, 4 = nibble
+                           (RF_AN only, else TQ_ERR_UNSUPPORTED); other
+                           values TQ_ERR_INVALID                            */
+    int deep_grid;      /* threads == 0 only: 0 = default on (after a run of
+                           >= 1,024 levels later runs use one block per SM),
+                           < 0 = always the full persistent grid            */
+    int l2_persist;     /* 0 = default on: the level mirror is launched with a
+                           persisting-L2 access-policy window (the device's
+                           persisting limit is raised while any such plan
+                           exists, shared by reference count); < 0 = off    */
 } bfs_opts;
 
 enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };
@@ -241,6 +260,16 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
                              int32_t *level_out, int32_t *parent_out, int64_t out_stride,
                              bfs_stats *stats);
 tq_status bfs_plan_destroy(bfs_plan *p);
+/* Restart the plan's queues at the given tickets (tq_reset_at on the main
+ * queue at t_main and on the chunk queue, if the plan has one, at t_chunk);
+ * later runs continue from there.  For tests of the ticket arithmetic across
+ * the 2^32 wrap of the 32-bit sequence tags: a benchmark plan reaches ~5e10
+ * tickets after 1,600 scale-26 runs.  Not while a run is in flight
+ * (TQ_ERR_INVALID); t_main, t_chunk < 2^62. */
+tq_status bfs_plan_set_tickets(bfs_plan *p, uint64_t t_main, uint64_t t_chunk);
+/* Current tickets (the main queue's Rear where the next run starts, and the
+ * chunk queue's), for the same tests. */
+tq_status bfs_plan_get_tickets(const bfs_plan *p, uint64_t *t_main, uint64_t *t_chunk);
 
 /* ------------------------------------------------------------------------ */
 /* The queue as a generic scheduler (NEXT row 4; "it can be used for    */

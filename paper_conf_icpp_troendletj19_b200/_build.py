@@ -55,3 +55,16 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
 if __name__ == "__main__":
     import sys
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+
+
+def build_user_kernel(src: str, out: str, force: bool = False) -> str:
+    """Build a standalone user-kernel library against the public headers
+    (include/tq.h, include/tq_device.cuh) -- e.g. the device-API test kernel
+    tests/csrc/devapi_test.cu -> tests/libtqdevapi.so."""
+    inputs = [src] + glob.glob(os.path.join(ROOT, "include", "*"))
+    if not force and up_to_date(out, inputs):
+        return out
+    tmp = out + f".tmp{os.getpid()}"
+    subprocess.check_call([NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), "-o", tmp, src])
+    os.replace(tmp, out)
+    return out

@@ -41,7 +41,8 @@ class bfs_opts(ctypes.Structure):
                 ("chunk", ctypes.c_int), ("variant", ctypes.c_int), ("stream", c_vp),
                 ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int),
                 ("parent_rule", ctypes.c_int), ("hub_queue", ctypes.c_int),
-                ("debug_delay_ns", ctypes.c_int), ("debug_delay_seed", c_u32)]
+                ("debug_delay_ns", ctypes.c_int), ("debug_delay_seed", c_u32),
+                ("mirror_bits", ctypes.c_int), ("deep_grid", ctypes.c_int), ("l2_persist", ctypes.c_int)]
 
 
 class bfs_stats(ctypes.Structure):
@@ -73,6 +74,7 @@ EXPORTS = {
     "tq_create": (ctypes.c_int, [c_u64, ctypes.c_int, ctypes.POINTER(c_vp)]),
     "tq_destroy": (ctypes.c_int, [c_vp]),
     "tq_reset": (ctypes.c_int, [c_vp, c_vp]),
+    "tq_reset_at": (ctypes.c_int, [c_vp, c_u64, c_vp]),
     "tq_device_view_get": (ctypes.c_int, [c_vp, ctypes.POINTER(tq_device_view)]),
     "tq_counters_get": (ctypes.c_int, [c_vp, ctypes.POINTER(tq_counters)]),
     "bfs_run": (ctypes.c_int, [ctypes.POINTER(tq_csr), c_i32, c_vp, c_vp]),
@@ -82,6 +84,8 @@ EXPORTS = {
                                        ctypes.POINTER(c_vp)]),
     "bfs_plan_run": (ctypes.c_int, [c_vp, c_i32, c_vp, c_vp, ctypes.POINTER(bfs_stats)]),
     "bfs_plan_destroy": (ctypes.c_int, [c_vp]),
+    "bfs_plan_set_tickets": (ctypes.c_int, [c_vp, c_u64, c_u64]),
+    "bfs_plan_get_tickets": (ctypes.c_int, [c_vp, ctypes.POINTER(c_u64), ctypes.POINTER(c_u64)]),
     "bfs_plan_launch": (ctypes.c_int, [c_vp, c_i32, c_vp, c_vp]),
     "bfs_plan_wait": (ctypes.c_int, [c_vp, ctypes.POINTER(bfs_stats)]),
     "bfs_plan_run_batch": (ctypes.c_int, [c_vp, c_vp, c_i32, c_vp, c_vp, c_i64, c_vp]),

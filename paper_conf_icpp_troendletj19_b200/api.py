@@ -75,11 +75,17 @@ def _csr(row_ptr, col) -> _lib.tq_csr:
 
 def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None, timeout_s=0.0,
           backoff_ns=0, device=0, parents="any", hub_queue=True, debug_delay_ns=0,
-          debug_delay_seed=0) -> _lib.bfs_opts:
+          debug_delay_seed=0, mirror_bits=0, deep_grid=True, l2_persist=True) -> _lib.bfs_opts:
     return _lib.bfs_opts(int(capacity), int(threads), int(block), int(chunk), _variant(variant),
                          stream, float(timeout_s), int(backoff_ns), int(device),
                          _lib.PARENT_RULES[parents] if isinstance(parents, str) else int(parents),
-                         0 if hub_queue else -1, int(debug_delay_ns), int(debug_delay_seed) & 0xFFFFFFFF)
+                         0 if hub_queue else -1, int(debug_delay_ns), int(debug_delay_seed) & 0xFFFFFFFF,
+                         int(mirror_bits), 0 if deep_grid else -1, 0 if l2_persist else -1)
+
+
+# bfs / BfsPlan keyword options that map one to one onto bfs_opts fields
+_OPT_KEYS = ("variant", "capacity", "threads", "chunk", "timeout_s", "backoff_ns", "parents", "hub_queue",
+             "debug_delay_ns", "debug_delay_seed", "mirror_bits", "deep_grid", "l2_persist")
 
 
 def _stats_dict(st: _lib.bfs_stats) -> dict:
@@ -93,25 +99,27 @@ def _empty_like_graph(row_ptr, n):
     return np.empty(n, dtype=np.int32)
 
 
-def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool = True,
-        variant="rf_an", capacity: int = 0, threads: int = 0, chunk: int = 0, stream=None,
-        timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0, parents="any",
-        hub_queue: bool = True, debug_delay_ns: int = 0, debug_delay_seed: int = 0):
+def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool = True, stream=None,
+        device: int = 0, **opts):
     """One-shot `bfs_run_ex`: returns (level, parent, stats).
 
     Graph arrays may be CUDA tensors (used in place) or host numpy arrays
     (staged to the device by the library). Outputs default to the graph's
-    kind of memory.
+    kind of memory. `opts`: the bfs_opts fields (variant, capacity, threads,
+    chunk, timeout_s, backoff_ns, parents, hub_queue, debug_delay_ns,
+    debug_delay_seed, mirror_bits, deep_grid, l2_persist).
     """
+    bad = set(opts) - set(_OPT_KEYS)
+    if bad:
+        raise TypeError(f"unknown options {sorted(bad)}")
     g = _csr(row_ptr, col)
     n = g.n_vertices
     if level is None:
         level = _empty_like_graph(row_ptr, n)
     if parent is None and want_parent:
         parent = _empty_like_graph(row_ptr, n)
-    o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr), timeout_s,
-              backoff_ns, row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device,
-              parents, hub_queue, debug_delay_ns, debug_delay_seed)
+    o = _opts(stream=_stream_ptr(stream, row_ptr),
+              device=row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device, **opts)
     st = _lib.bfs_stats()
     check(lib().bfs_run_ex(ctypes.byref(g), int(root), _ptr(level), _ptr(parent), ctypes.byref(o),
                            ctypes.byref(st)), "bfs_run_ex")
@@ -125,18 +133,16 @@ class BfsPlan:
     chunk table live for the plan's lifetime; `run` only launches.
     """
 
-    def __init__(self, row_ptr, col, *, variant="rf_an", capacity: int = 0, threads: int = 0,
-                 chunk: int = 0, stream=None, timeout_s: float = 0.0, backoff_ns: int = 0,
-                 device: int = 0, parents="any", hub_queue: bool = True, debug_delay_ns: int = 0,
-                 debug_delay_seed: int = 0):
+    def __init__(self, row_ptr, col, *, stream=None, device: int = 0, **opts):
+        bad = set(opts) - set(_OPT_KEYS)
+        if bad:
+            raise TypeError(f"unknown options {sorted(bad)}")
         self._keep = (row_ptr, col)  # device arrays must outlive the plan
         self._g = _csr(row_ptr, col)
         self.n_vertices = self._g.n_vertices
         self.nnz = self._g.nnz
         self.device = row_ptr.device.index if _is_tensor(row_ptr) and row_ptr.is_cuda else device
-        self._opts = o = _opts(variant, capacity, threads, 0, chunk, _stream_ptr(stream, row_ptr),
-                               timeout_s, backoff_ns, self.device, parents, hub_queue, debug_delay_ns,
-                               debug_delay_seed)
+        self._opts = _opts(stream=_stream_ptr(stream, row_ptr), device=self.device, **opts)
         self.regrows = 0
         self._h = None
         self._create()
@@ -147,22 +153,48 @@ class BfsPlan:
               "bfs_plan_create")
         self._h = h
 
+    # the largest queue the library builds (tq_create: C <= 2^31)
+    MAX_CAPACITY = 1 << 31
+    MAX_REGROWS = 12
+
+    def _grow(self) -> bool:
+        """Queue-full answer of the paper: re-create the plan with
+        twice the queue capacity (the chunk queue follows it). False once the
+        capacity cannot grow any more or MAX_REGROWS retries were spent."""
+        cap = self._opts.capacity or 2 * max(self.n_vertices, 1 << 15)
+        new = min(2 * max(cap, 1 << 16), self.MAX_CAPACITY)
+        if new <= (self._opts.capacity or 0) or self.regrows >= self.MAX_REGROWS:
+            return False
+        self._opts.capacity = new
+        self.close()
+        self._create()
+        self.regrows += 1
+        return True
+
     def run(self, root: int, level=None, parent=None, grow_on_full: bool = False) -> dict:
         """One BFS. With grow_on_full, a queue-full abort (TQ_ERR_QUEUE_FULL)
         is answered as the paper suggests: re-create the plan with
-        twice the queue capacity and run again (counted in `regrows`)."""
+        twice the queue capacity and run again (counted in `regrows`), at most
+        MAX_REGROWS times and never past MAX_CAPACITY; then the error is raised."""
         while True:
             st = _lib.bfs_stats()
             status = lib().bfs_plan_run(self._h, int(root), _ptr(level), _ptr(parent), ctypes.byref(st))
-            if status == _lib.TQ_ERR_QUEUE_FULL and grow_on_full:
-                cap = self._opts.capacity or 2 * max(self.n_vertices, 1 << 15)
-                self._opts.capacity = 2 * max(cap, 1 << 16)
-                self.close()
-                self._create()
-                self.regrows += 1
+            if status == _lib.TQ_ERR_QUEUE_FULL and grow_on_full and self._grow():
                 continue
             check(status, "bfs_plan_run")
             return _stats_dict(st)
+
+    def set_tickets(self, t_main: int, t_chunk: int = 0):
+        """`bfs_plan_set_tickets`: restart the queues at these tickets (tests of
+        the 32-bit sequence-tag wrap)."""
+        check(lib().bfs_plan_set_tickets(self._h, int(t_main), int(t_chunk)), "bfs_plan_set_tickets")
+
+    def tickets(self) -> tuple:
+        """`bfs_plan_get_tickets`: (main-queue ticket, chunk-queue ticket) where
+        the next run starts."""
+        a, b = ctypes.c_uint64(), ctypes.c_uint64()
+        check(lib().bfs_plan_get_tickets(self._h, ctypes.byref(a), ctypes.byref(b)), "bfs_plan_get_tickets")
+        return a.value, b.value
 
     def run_batch(self, roots, level=None, parent=None, stride: int | None = None) -> list:
         """`bfs_plan_run_batch`: root i writes level[i * stride:] / parent[...].
@@ -213,14 +245,10 @@ class SsspPlan(BfsPlan):
     the same queue and persistent kernel (include/tq.h, NEXT row 4). `weights`
     is int32[nnz] (>= 1), host or device like the CSR."""
 
-    def __init__(self, row_ptr, col, weights, *, capacity: int = 0, threads: int = 0, chunk: int = 0,
-                 stream=None, timeout_s: float = 0.0, backoff_ns: int = 0, device: int = 0,
-                 hub_queue: bool = True, debug_delay_ns: int = 0, debug_delay_seed: int = 0):
+    def __init__(self, row_ptr, col, weights, *, stream=None, device: int = 0, **opts):
         self._w = weights
-        super().__init__(row_ptr, col, variant="rf_an", capacity=capacity, threads=threads, chunk=chunk,
-                         stream=stream, timeout_s=timeout_s, backoff_ns=backoff_ns, device=device,
-                         parents="min_id", hub_queue=hub_queue, debug_delay_ns=debug_delay_ns,
-                         debug_delay_seed=debug_delay_seed)
+        opts = dict(opts, variant="rf_an", parents="min_id")
+        super().__init__(row_ptr, col, stream=stream, device=device, **opts)
 
     def _create(self):
         h = ctypes.c_void_p()
@@ -233,12 +261,7 @@ class SsspPlan(BfsPlan):
         while True:
             st = _lib.bfs_stats()
             status = lib().sssp_plan_run(self._h, int(src), _ptr(dist), _ptr(parent), ctypes.byref(st))
-            if status == _lib.TQ_ERR_QUEUE_FULL and grow_on_full:
-                cap = self._opts.capacity or 2 * max(self.n_vertices, 1 << 15)
-                self._opts.capacity = 2 * max(cap, 1 << 16)
-                self.close()
-                self._create()
-                self.regrows += 1
+            if status == _lib.TQ_ERR_QUEUE_FULL and grow_on_full and self._grow():
                 continue
             check(status, "sssp_plan_run")
             return _stats_dict(st)
@@ -286,6 +309,10 @@ class Queue:
 
     def reset(self, stream=None):
         check(lib().tq_reset(self._h, stream), "tq_reset")
+
+    def reset_at(self, ticket: int, stream=None):
+        """`tq_reset_at`: empty queue with Front = Rear = Done = ticket."""
+        check(lib().tq_reset_at(self._h, int(ticket), stream), "tq_reset_at")
 
     def view(self) -> _lib.tq_device_view:
         v = _lib.tq_device_view()

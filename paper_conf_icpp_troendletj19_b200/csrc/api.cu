@@ -135,13 +135,15 @@ tq_status from_cuda(cudaError_t e)
         if (e_ != cudaSuccess) return from_cuda(e_);    \
     } while (0)
 
-// Returns 1 for device (or managed) memory, 0 for host memory, -1 on error.
+// Returns 1 for device (or managed) memory, 0 for host memory (pageable or
+// pinned), -1 when the pointer cannot be classified (the query failed: the
+// entry points then return TQ_ERR_INVALID instead of guessing).
 int is_device_ptr(const void *p, int *device)
 {
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
         cudaGetLastError();
-        return 0;
+        return -1;
     }
     if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
         if (device) *device = a.device;
@@ -165,6 +167,73 @@ static cudaError_t d2h_chunked(void *dst, const void *src, size_t bytes, cudaStr
         if (e != cudaSuccess) return e;
     }
     return cudaSuccess;
+}
+
+// Persisting-L2 carve-out: the limit is device-wide, the windows are per
+// launch.  Plans on one device share it through a reference count, so
+// destroying one plan never resets the persisting lines of another plan that
+// is still running (e.g. run_concurrent); the limit is raised by the first
+// plan that needs it and restored, and the persisting lines reset, when the
+// last plan on the device is destroyed.
+struct L2Persist {
+    int refs = 0;
+    size_t saved = 0;   // device limit before the first plan raised it
+    size_t cur = 0;     // limit now
+    bool raised = false;
+};
+static L2Persist g_l2[256];
+static std::mutex g_l2_mu;
+
+// Returns the window size to use for `want` bytes (0 = no window); every
+// non-zero return must be paired with one l2_persist_release(dev).
+size_t l2_persist_acquire(int dev, size_t want)
+{
+    std::lock_guard<std::mutex> lk(g_l2_mu);
+    if (dev < 0 || dev >= 256 || want == 0) return 0;
+    int max_win = 0, max_persist = 0;
+    cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+    cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, dev);
+    size_t w = want;
+    if (w > (size_t)max_win) w = (size_t)max_win;
+    if (w > (size_t)max_persist) w = (size_t)max_persist;
+    if (w == 0) {
+        cudaGetLastError();
+        return 0;
+    }
+    L2Persist &e = g_l2[dev];
+    if (e.refs == 0) {
+        size_t cur = 0;
+        if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) != cudaSuccess) {
+            cudaGetLastError();
+            return 0;
+        }
+        e.saved = e.cur = cur;
+        e.raised = false;
+    }
+    if (e.cur < w) {
+        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, w) == cudaSuccess) {
+            e.cur = w;
+            e.raised = true;
+        } else {
+            cudaGetLastError();
+        }
+    }
+    ++e.refs;
+    return w;
+}
+
+void l2_persist_release(int dev)
+{
+    std::lock_guard<std::mutex> lk(g_l2_mu);
+    if (dev < 0 || dev >= 256) return;
+    L2Persist &e = g_l2[dev];
+    if (e.refs <= 0) return;
+    if (--e.refs == 0) {
+        cudaCtxResetPersistingL2Cache();
+        if (e.raised) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, e.saved);
+        e.raised = false;
+        cudaGetLastError();
+    }
 }
 
 uint64_t next_pow2(uint64_t x)
@@ -231,8 +300,6 @@ struct bfs_plan {
     cudaStream_t copy_stream = nullptr;       // batch: D2H copies
     cudaEvent_t bfs_done[2] = {nullptr, nullptr}, copy_done[2] = {nullptr, nullptr};
     size_t l2_window = 0;                     // persisting-L2 window over the level mirror
-    size_t l2_limit_saved = 0;                // device persisting-L2 limit to restore
-    bool l2_limit_set = false;
     unsigned long long next_ticket = 0;
     bool dirty = false;
     int32_t *out_scratch = nullptr;           // for host outputs
@@ -335,14 +402,16 @@ tq_status tq_destroy(tq_queue *q)
     return TQ_OK;
 }
 
-tq_status tq_reset(tq_queue *q, void *stream)
+tq_status tq_reset_at(tq_queue *q, uint64_t t0, void *stream)
 {
-    if (!q) return TQ_ERR_INVALID;
+    if (!q || t0 >= (1ull << 63)) return TQ_ERR_INVALID;
     DeviceGuard g(q->device);
     CK(cudaMemsetAsync(q->ctr, 0, kCtrBytes, (cudaStream_t)stream));
-    CK(launch_queue_reset(q->view, (cudaStream_t)stream));
+    CK(launch_queue_reset(q->view, t0, (cudaStream_t)stream));
     return TQ_OK;
 }
+
+tq_status tq_reset(tq_queue *q, void *stream) { return tq_reset_at(q, 0, stream); }
 
 tq_status tq_device_view_get(const tq_queue *q, tq_device_view *out)
 {
@@ -389,22 +458,10 @@ tq_status bfs_plan_destroy(bfs_plan *p)
 {
     if (!p) return TQ_OK;
     DeviceGuard g(p->device);
-    // TQ_DEBUG_DESTROY=1: per-step timing to stderr (diagnostics only)
-    const bool dbg = getenv("TQ_DEBUG_DESTROY") != nullptr;
-    double tt[8] = {0};
-    int ti = 0;
-    auto tick = [&]() {
-        if (!dbg) return;
-        timespec ts;
-        clock_gettime(CLOCK_MONOTONIC, &ts);
-        tt[ti++] = ts.tv_sec + ts.tv_nsec * 1e-9;
-    };
-    tick();
     if (p->stream) cudaStreamSynchronize(p->stream);
     for (auto &e : p->ev)
         if (e) cudaEventDestroy(e);
     if (p->copy_stream) cudaStreamSynchronize(p->copy_stream);
-    tick();
     // stream-ordered frees after everything that used the memory has finished
     cudaStream_t fs = p->stream;
     if (p->owns_graph) {
@@ -425,21 +482,12 @@ tq_status bfs_plan_destroy(bfs_plan *p)
         if (p->bfs_done[b]) cudaEventDestroy(p->bfs_done[b]);
         if (p->copy_done[b]) cudaEventDestroy(p->copy_done[b]);
     }
-    tick();
     if (p->copy_stream) cudaStreamDestroy(p->copy_stream);
     pinned_small_free(p->stats_h);
     pinned_small_free(p->ctr_h);
-    tick();
-    if (p->l2_window) cudaCtxResetPersistingL2Cache();
-    tick();
-    if (p->l2_limit_set) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, p->l2_limit_saved);
-    tick();
+    if (p->l2_window) l2_persist_release(p->device);
     tq_destroy(p->q);
     tq_destroy(p->q1);
-    tick();
-    if (dbg)
-        fprintf(stderr, "TQDESTROY sync %.4f frees %.4f host %.4f l2reset %.4f l2limit %.4f queues %.4f\n",
-                tt[1] - tt[0], tt[2] - tt[1], tt[3] - tt[2], tt[4] - tt[3], tt[5] - tt[4], tt[6] - tt[5]);
     delete p;
     return TQ_OK;
 }
@@ -465,7 +513,9 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
 
     int gdev = o.device;
     const int dev_graph = is_device_ptr(gph->row_ptr, &gdev);
-    if (dev_graph && nnz > 0 && !is_device_ptr(gph->col, nullptr)) return TQ_ERR_INVALID;
+    if (dev_graph < 0) return TQ_ERR_INVALID;
+    if (nnz > 0 && is_device_ptr(gph->col, nullptr) != dev_graph) return TQ_ERR_INVALID;  // same kind
+    if (o.mirror_bits != 0 && o.mirror_bits != 4 && o.mirror_bits != 8) return TQ_ERR_INVALID;
     DeviceGuard g(gdev);
     if (!g.ok) return TQ_ERR_INVALID;
 
@@ -514,7 +564,9 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         if (e != cudaSuccess) return fail(from_cuda(e));
     }
     if (task == kTaskSSSP && nnz > 0) {
-        if (is_device_ptr(weights, nullptr)) {
+        const int wdev = is_device_ptr(weights, nullptr);
+        if (wdev < 0) return fail(TQ_ERR_INVALID);
+        if (wdev) {
             p->wgt = const_cast<int32_t *>(weights);
         } else {
             p->owns_wgt = true;
@@ -531,10 +583,10 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         // Level mirror width (R8): a nibble per vertex when a byte
         // mirror would exceed 32 MB (it then no longer stays L2-resident next
         // to the col stream; measured: s26 -3.6%, s24 / grid +2-4% with
-        // nibbles), RF/AN only.  TQ_MIRROR_BITS=4|8 overrides (experiments).
+        // nibbles), RF/AN only.  bfs_opts.mirror_bits overrides.
         p->mirror_bits = (o.variant == TQ_VARIANT_RF_AN && n > (1ll << 25)) ? 4 : 8;
-        const char *mb = getenv("TQ_MIRROR_BITS");
-        if (mb && o.variant == TQ_VARIANT_RF_AN && (mb[0] == '4' || mb[0] == '8')) p->mirror_bits = mb[0] - '0';
+        if (o.mirror_bits == 4 || o.mirror_bits == 8) p->mirror_bits = o.mirror_bits;
+        if (p->mirror_bits == 4 && o.variant != TQ_VARIANT_RF_AN) return fail(TQ_ERR_UNSUPPORTED);
         p->mirror_bytes = p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 7) / 8 * 4;
         if (e == cudaSuccess) e = pool_alloc(&p->mir, p->mirror_bytes, p->stream);
         // expanded-level markers: same width as the mirror
@@ -562,12 +614,20 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     if (st != TQ_OK) return fail(st);
     // chunk queue (RF/AN only): a hub emits its chunks at every expansion
     // (one per distinct level, R7); 4x the chunk count, at least 2^20 slots
-    // (8 MiB), leaves room for bursts while consumers lag (e.g. under ncu)
+    // (8 MiB), leaves room for bursts while consumers lag (e.g. under ncu).
+    // An explicit capacity C bounds it by C and raises it to at least C/4, so
+    // a caller that answers a queue-full abort by doubling C (the
+    // Python binding's grow_on_full) also grows the chunk queue.
     p->hub_queue = p->variant == TQ_VARIANT_RF_AN && o.hub_queue >= 0 && p->n_chunks > 0;
     if (p->hub_queue) {
         uint64_t cap1 = next_pow2((uint64_t)(4 * p->n_chunks));
         if (cap1 < (1ull << 20)) cap1 = 1ull << 20;
-        if (o.capacity && cap1 > next_pow2(o.capacity)) cap1 = next_pow2(o.capacity);
+        if (o.capacity) {
+            const uint64_t c = next_pow2(o.capacity);
+            if (cap1 > c) cap1 = c;
+            if (cap1 < c / 4) cap1 = c / 4;
+            if (cap1 < 2) cap1 = 2;
+        }
         st = tq_create(cap1, gdev, &p->q1);
         if (st != TQ_OK) return fail(st);
     }
@@ -580,30 +640,15 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         p->blocks = (o.threads + p->block - 1) / p->block;
     } else {
         p->blocks = full;
-        p->auto_blocks = task == kTaskBFS && !getenv("TQ_NO_DEEP_GRID");
+        p->auto_blocks = task == kTaskBFS && o.deep_grid >= 0;
     }
     if (p->blocks < 1) p->blocks = 1;
-    const char *l2env = getenv("TQ_L2_WINDOW");  // "0": experiments only
-    if (task == kTaskBFS && !(l2env && l2env[0] == '0')) {
-        // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the byte
+    if (task == kTaskBFS && o.l2_persist >= 0) {
+        // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the level
         // mirror is probed once per edge; a persisting window keeps it
-        // resident against the col stream.  The device-wide carve-out is
-        // raised here if needed and restored by bfs_plan_destroy.
-        int max_win = 0, max_persist = 0;
-        cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, gdev);
-        cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, gdev);
-        size_t w = p->mirror_bytes;
-        if (w > (size_t)max_win) w = (size_t)max_win;
-        if (w > (size_t)max_persist) w = (size_t)max_persist;
-        size_t cur = 0;
-        if (w > 0 && cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
-            if (cur < w && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, w) == cudaSuccess) {
-                p->l2_limit_saved = cur;
-                p->l2_limit_set = true;
-            }
-            p->l2_window = w;
-        }
-        cudaGetLastError();
+        // resident against the col stream (shared device limit, see
+        // l2_persist_acquire)
+        p->l2_window = l2_persist_acquire(gdev, p->mirror_bytes);
     }
     e = cudaStreamSynchronize(p->stream);
     if (e != cudaSuccess) return fail(from_cuda(e));
@@ -735,12 +780,6 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
         stats->busy_cycles = h[ST_BUSY_CYCLES];
         stats->rounds = h[ST_ROUNDS];
         stats->persistent_threads = p->blocks * p->block;
-#ifdef TQ_AB_PROF
-        fprintf(stderr, "TQPROF idle %.4g prolog %.4g expand %.4g enqueue %.4g | in rounds: col %.4g probe %.4g "
-                "mid %.4g atomic+stage %.4g (SM cycles, summed over warps)\n",
-                (double)h[16], (double)h[17], (double)h[18], (double)h[19], (double)h[20], (double)h[21],
-                (double)(h[18] - h[20] - h[21] - h[22]), (double)h[22]);
-#endif
     }
     // Deep graphs: a BFS of >= 1,024 levels runs a few thousand
     // vertices per level at a time; a full persistent grid then spends L2 on
@@ -757,11 +796,33 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
     return TQ_ERR_CUDA;
 }
 
+tq_status bfs_plan_set_tickets(bfs_plan *p, uint64_t t_main, uint64_t t_chunk)
+{
+    if (!p || p->in_flight || t_main >= (1ull << 62) || t_chunk >= (1ull << 62)) return TQ_ERR_INVALID;
+    DeviceGuard g(p->device);
+    tq_status st = tq_reset_at(p->q, t_main, p->stream);
+    if (st == TQ_OK && p->q1) st = tq_reset_at(p->q1, t_chunk, p->stream);
+    if (st == TQ_OK) st = from_cuda(cudaStreamSynchronize(p->stream));
+    if (st != TQ_OK) return st;
+    p->next_ticket = t_main;
+    p->next_ticket1 = p->q1 ? t_chunk : 0;
+    p->dirty = false;
+    return TQ_OK;
+}
+
+tq_status bfs_plan_get_tickets(const bfs_plan *p, uint64_t *t_main, uint64_t *t_chunk)
+{
+    if (!p || !t_main || !t_chunk) return TQ_ERR_INVALID;
+    *t_main = p->next_ticket;
+    *t_chunk = p->next_ticket1;
+    return TQ_OK;
+}
+
 tq_status bfs_plan_launch(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out)
 {
     if (!p || root < 0 || root >= p->n) return TQ_ERR_INVALID;
-    if ((level_out && !is_device_ptr(level_out, nullptr)) ||
-        (parent_out && !is_device_ptr(parent_out, nullptr)))
+    if ((level_out && is_device_ptr(level_out, nullptr) != 1) ||
+        (parent_out && is_device_ptr(parent_out, nullptr) != 1))
         return TQ_ERR_INVALID;  // the asynchronous form takes device outputs only
     DeviceGuard g(p->device);
     return plan_launch(p, root, level_out, parent_out);
@@ -782,8 +843,10 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
     for (int32_t i = 0; i < n_roots; ++i)
         if (roots[i] < 0 || roots[i] >= p->n) return TQ_ERR_INVALID;
     DeviceGuard g(p->device);
-    const bool host_l = level_out && !is_device_ptr(level_out, nullptr);
-    const bool host_p = parent_out && !is_device_ptr(parent_out, nullptr);
+    const int kind_l = level_out ? is_device_ptr(level_out, nullptr) : 1;
+    const int kind_p = parent_out ? is_device_ptr(parent_out, nullptr) : 1;
+    if (kind_l < 0 || kind_p < 0) return TQ_ERR_INVALID;
+    const bool host_l = kind_l == 0, host_p = kind_p == 0;
     const size_t vb = (size_t)p->n * sizeof(int32_t);
     if (host_l || host_p) {
         // two device output pairs + a copy stream, allocated on first use
@@ -844,8 +907,10 @@ tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *p
 {
     if (!p || root < 0 || root >= p->n) return TQ_ERR_INVALID;
     DeviceGuard g(p->device);
-    const bool host_l = level_out && !is_device_ptr(level_out, nullptr);
-    const bool host_p = parent_out && !is_device_ptr(parent_out, nullptr);
+    const int kind_l = level_out ? is_device_ptr(level_out, nullptr) : 1;
+    const int kind_p = parent_out ? is_device_ptr(parent_out, nullptr) : 1;
+    if (kind_l < 0 || kind_p < 0) return TQ_ERR_INVALID;
+    const bool host_l = kind_l == 0, host_p = kind_p == 0;
     if (!host_l && !host_p) {
         const tq_status st = plan_launch(p, root, level_out, parent_out);
         return st == TQ_OK ? plan_finish(p, stats) : st;

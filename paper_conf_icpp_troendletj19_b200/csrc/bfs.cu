@@ -32,12 +32,6 @@ namespace tqk {
 
 constexpr int kBlock = 256;          // threads per block (8 warps)
 constexpr int kWarps = kBlock / 32;
-#ifndef TQ_AB_STAGE
-#define TQ_AB_STAGE 512
-#endif
-#ifndef TQ_AB_STAGE_BYTE
-#define TQ_AB_STAGE_BYTE 768
-#endif
 // Staged tokens per warp (2-3 KiB smem). A larger stage publishes children in
 // bigger, later batches: fewer label-correcting re-scans, less work visible to
 // idle warps. Measured (results/ab_occupancy_r01.md, stage sweeps): 768 is best
@@ -47,23 +41,15 @@ constexpr int kWarps = kBlock / 32;
 // spread, 18.6-25.4 ms per s24 source at either size, hides any difference).
 template <int MIR, int TASK> __host__ __device__ constexpr int stage_cap()
 {
-    return (MIR == 8 && TASK == kTaskBFS) ? TQ_AB_STAGE_BYTE : TQ_AB_STAGE;
+    return (MIR == 8 && TASK == kTaskBFS) ? 768 : 512;
 }
-// A/B builds (scripts/ab_bfs.py) override these with -D; the defaults are
-// the measured best.
-#ifndef TQ_AB_KU
-#define TQ_AB_KU 4
-#endif
-#ifndef TQ_AB_MINB
-#define TQ_AB_MINB 5
-#endif
-constexpr int kU = TQ_AB_KU;         // 32-edge rounds in flight per lane
+constexpr int kU = 4;                // 32-edge rounds in flight per lane
 // Resident blocks per SM requested from ptxas (40 warps/SM; <= 48 registers).
 // The expansion is bound by the L2 request rate of its random mirror probes
 // (DESIGN.md section 6), so occupancy matters through latency hiding and
 // spills; interleaved A/B on B200 (results/ab_occupancy_r01.md): 5 blocks
 // beat 6 by 1-3% on Kronecker and 8% on the grid, 4 and 8 blocks are slower.
-constexpr int kMinBlocks = TQ_AB_MINB;
+constexpr int kMinBlocks = 5;
 constexpr unsigned kLvlSat = 254;    // byte: 0..253 exact, 254 = ">= 254", 255 = unreached / none
 // Level mirror (R8), MIR bits per vertex:
 //   MIR = 8: one byte per vertex: 0..253 exact-or-stale-high, 254 = ">= 254",
@@ -127,15 +113,6 @@ __device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long lon
     asm volatile("ld.global.cg.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
-#ifdef TQ_AB_L1PROBE
-#define ld_cg_u8 ld_ca_u8
-__device__ __forceinline__ unsigned ld_ca_u8(const uint8_t *p, unsigned long long pol)
-{
-    unsigned v;
-    asm volatile("ld.global.ca.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-    return v;
-}
-#endif
 __device__ __forceinline__ unsigned mix32(unsigned x)
 {
     x ^= x >> 16;
@@ -419,6 +396,11 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
             base = tq_warp_reserve_rear(q, n, qatom);
         } else if constexpr (VARIANT == TQ_VARIANT_AN) {
             if (!an_reserve_rear(q, n, &base, qatom, casfail)) return;
+        }
+        if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
+            // release: a chunk token names the hub's W entry (its level), and
+            // this warp's Rear reservation is ordered before its Done increment
+            tq_fence_release();
         } else {  // PER_THREAD_AFA: each lane reserves its own share
             const unsigned mine = lane < n ? (n - lane + 31) / 32 : 0;
             base = 0;
@@ -510,15 +492,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         }
     }
 
-#ifdef TQ_AB_PROF
-#define TQ_PROF_T(v) long long v = clock64()
-#define TQ_PROF_ADD(k, d) do { if (lane == 0) S[16 + (k)] += (unsigned long long)(d); } while (0)
-#else
-#define TQ_PROF_T(v)
-#define TQ_PROF_ADD(k, d)
-#endif
     for (;;) {
-        TQ_PROF_T(t0);
         // ---- Listing 1 + Listing 2: GetWorkToken() ----
         bool got = false, got1 = false;
         uint32_t item = 0;
@@ -549,15 +523,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             // lane issues both polls back to back and prefers the chunk
             // (acquire loads: a hit makes the producer's W update visible,
             // with no fence; ld.acquire.gpu is LDG.STRONG.GPU + CCTL.IVALL)
-#ifdef TQ_AB_L1PROBE
-            const unsigned long long sv0 = have ? tq_ld_relaxed(q.slots + (tk & q.mask)) : 0ull;
-            const unsigned long long sv1 =
-                (q1_lane && have1) ? tq_ld_relaxed(q1.slots + (tk1 & q1.mask)) : 0ull;
-#else
             const unsigned long long sv0 = have ? tq_ld_acquire(q.slots + (tk & q.mask)) : 0ull;
             const unsigned long long sv1 =
                 (q1_lane && have1) ? tq_ld_acquire(q1.slots + (tk1 & q1.mask)) : 0ull;
-#endif
             got1 = q1_lane && have1 && (unsigned)sv1 == tk1 + 1u;
             got = !got1 && have && (unsigned)sv0 == tk + 1u;
             item = (uint32_t)((got1 ? sv1 : sv0) >> 32);
@@ -603,24 +571,17 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 backoff = backoff ? min(backoff * 2, (unsigned)p.backoff_ns) : 32u;
                 __nanosleep(backoff);
             }
-            TQ_PROF_ADD(0, clock64() - t0);
             continue;
         }
         backoff = 0;
         idle = 0;
-#ifdef TQ_AB_L1PROBE
-#ifndef TQ_AB_L1REFRESH
-#define TQ_AB_L1REFRESH 63
-#endif
-        if (((++busy) & TQ_AB_L1REFRESH) == 0) {
-            unsigned stv;
-            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(stv)
-                         : "l"(q.status + (warp_gid % TQ_STATUS_COPIES) * TQ_STATUS_STRIDE) : "memory");
-            if (stv != TQ_RUNNING) break;
+        if (((++busy) & 63) == 0) {
+            if (tq_status_read(q, warp_gid) != TQ_RUNNING) break;
+            // the watchdog is honoured by busy warps too: a livelock that keeps
+            // every warp busy never reaches the idle-path check
+            if ((busy & 1023) == 0 && lane == 0 && tq_globaltimer() > wdeadline[threadIdx.x >> 5])
+                tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
         }
-#else
-        if (((++busy) & 63) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
-#endif
         if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY || VARIANT == TQ_VARIANT_AN)
             tq_fence_gpu();  // acquire for the comparators' relaxed dequeues
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
@@ -732,8 +693,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
         }
 
-        TQ_PROF_T(t1);
-        TQ_PROF_ADD(1, t1 - t0);
         // ---- DoWorkUnit(): warp-cooperative expansion ----
         const int deg = (int)(hi - lo);
         const int incl = warp_incl_scan(deg, lane);
@@ -765,10 +724,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             unsigned lv1[KU];            // BFS: offered level of each edge's token
             unsigned ownp = 0;           // BFS: owner lane of edge j in byte j
             bool val[KU];
-#ifdef TQ_AB_PROF
-            long long ta;
-            asm volatile("mov.u64 %0, %%clock64;" : "=l"(ta));
-#endif
 #pragma unroll
             for (int j = 0; j < KU; ++j) {
                 const int g = b + j * 32 + (int)lane;
@@ -788,11 +743,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     ownp |= (unsigned)o << (8 * j);
                 }
             }
-#ifdef TQ_AB_PROF
-            long long tb;  // after the col loads returned (the asm consumes them)
-            asm volatile("mov.u64 %0, %%clock64;" : "=l"(tb) : "r"(u[0]), "r"(u[KU - 1]), "r"(u[1]), "r"(u[2]));
-            TQ_PROF_ADD(4, tb - ta);
-#endif
             bool cand[KU];
             unsigned b8[KU];  // BFS: the probed mirror byte / word
             if constexpr (TASK == kTaskSSSP) {
@@ -818,11 +768,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     else
                         b8[j] = (val[j] && !deep) ? ld_cg_u32(p.mir + ((unsigned)u[j] >> 3), pol_keep) : ~0u;
                 }
-#ifdef TQ_AB_PROF
-                long long tc;  // after the mirror probes returned
-                asm volatile("mov.u64 %0, %%clock64;" : "=l"(tc) : "r"(b8[0]), "r"(b8[KU - 1]), "r"(b8[1]), "r"(b8[2]));
-                TQ_PROF_ADD(5, tc - tb);
-#endif
                 bool tie[KU];
                 bool any_tie = false;
 #pragma unroll
@@ -846,10 +791,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     }
                 }
             }
-#ifdef TQ_AB_PROF
-            long long td;
-            asm volatile("mov.u64 %0, %%clock64;" : "=l"(td));
-#endif
             if constexpr (TASK == kTaskBFS) {
                 // Candidates (a few percent of the edges) are compacted into
                 // the free tail of the staging buffer -- vertex ids at
@@ -949,23 +890,13 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 __syncwarp();
                 cnt = 0;
             }
-#ifdef TQ_AB_PROF
-            {
-                long long te;
-                asm volatile("mov.u64 %0, %%clock64;" : "=l"(te));
-                TQ_PROF_ADD(6, te - td);  // atomics + staging (+ flushes)
-            }
-#endif
         }
 
-        TQ_PROF_T(t2);
-        TQ_PROF_ADD(2, t2 - t1);
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
         enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end);
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
-        const bool hubm_any = hubm != 0;
         while (hubm) {
             const int h = __ffs(hubm) - 1;
             hubm &= hubm - 1;
@@ -980,15 +911,11 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         // it is ordered after this warp's Rear reservations; idle warps
         // compare Done with Rear.
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
-            // lane 0 issued every Rear reservation of this warp.  The release
-            // fence before publishing staged tokens already ordered them; only
-            // a cycle that ended with chunk reservations (published without
-            // a fence) needs a release on Done itself.
+            // lane 0 issued every Rear reservation of this warp, and the
+            // release fence that follows each reservation (staged tokens and
+            // chunk tokens alike) already ordered it before this increment.
             if (lane == 0) {
-                if (hubm_any)
-                    tq_red_add_release(q.done, (unsigned long long)__popc(gm));
-                else
-                    tq_red_add_relaxed(q.done, (unsigned long long)__popc(gm));
+                tq_red_add_relaxed(q.done, (unsigned long long)__popc(gm));
                 ++st_qatom;
             }
         } else {
@@ -999,7 +926,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 ++st_qatom;
             }
         }
-        TQ_PROF_ADD(3, clock64() - t2);
     }
 
     // ---- statistics (one atomic per counter per warp) ----
@@ -1012,9 +938,6 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         }
         __syncwarp();
         if (lane < ST_REACHED && S[lane]) atomicAdd(p.stats + lane, S[lane]);
-#ifdef TQ_AB_PROF
-        if (lane >= 16 && lane < 23) atomicAdd(p.stats + lane, S[lane]);
-#endif
     }
 }
 
@@ -1205,19 +1128,20 @@ __global__ void fill_chunks_kernel(const int64_t *row_ptr, int64_t n, int chunk,
     }
 }
 
-__global__ void queue_reset_kernel(tq_device_view q)
+// Slot i holds "empty" for the ticket t in [t0, t0 + C) with t mod C == i.
+__global__ void queue_reset_kernel(tq_device_view q, unsigned long long t0)
 {
     const unsigned long long cap = q.mask + 1;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < cap;
          i += stride)
-        q.slots[i] = (unsigned)i;  // empty for ticket i (lap 0)
+        q.slots[i] = (unsigned)(t0 + ((i - t0) & q.mask));
     if (blockIdx.x == 0) {
         if (threadIdx.x < TQ_STATUS_COPIES) q.status[threadIdx.x * TQ_STATUS_STRIDE] = TQ_RUNNING;
         if (threadIdx.x == 0) {
-            *q.front = 0;
-            *q.rear = 0;
-            *q.done = 0;
+            *q.front = t0;
+            *q.rear = t0;
+            *q.done = t0;
         }
     }
 }
@@ -1248,9 +1172,9 @@ cudaError_t launch_bfs_unpack(const BfsParams &p, int32_t *level, int32_t *paren
     return cudaGetLastError();
 }
 
-cudaError_t launch_queue_reset(const tq_device_view &q, cudaStream_t s)
+cudaError_t launch_queue_reset(const tq_device_view &q, unsigned long long t0, cudaStream_t s)
 {
-    queue_reset_kernel<<<grid_for((int64_t)(q.mask + 1), 256), 256, 0, s>>>(q);
+    queue_reset_kernel<<<grid_for((int64_t)(q.mask + 1), 256), 256, 0, s>>>(q, t0);
     return cudaGetLastError();
 }
 

@@ -42,11 +42,7 @@ inline cudaError_t pool_alloc(T **p, size_t bytes, cudaStream_t s)
     return pool_alloc_raw(reinterpret_cast<void **>(p), bytes, s);
 }
 
-#ifdef TQ_AB_PROF
-constexpr int kStatCount = 24;  // 16..19: idle / prolog / expand / enqueue SM cycles (A/B builds only)
-#else
 constexpr int kStatCount = 16;
-#endif
 
 // Task run by the persistent kernel over the queue (the queue is the same).
 constexpr int kTaskBFS = 0;   // top-down BFS levels (the paper's driver)
@@ -111,7 +107,7 @@ cudaError_t launch_bfs_unpack(const BfsParams &p, int32_t *level, int32_t *paren
 cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm);
 cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int32_t *hub_base,
                               int2 **chunk_tab_out, int64_t *n_chunks_out, cudaStream_t s);
-cudaError_t launch_queue_reset(const tq_device_view &q, cudaStream_t s);
+cudaError_t launch_queue_reset(const tq_device_view &q, unsigned long long t0, cudaStream_t s);
 
 // bench.cu
 struct BenchParams {

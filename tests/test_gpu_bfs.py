@@ -377,20 +377,19 @@ def test_plans_recycled_through_the_memory_pool(tq):
     tq.memory_trim(0)
 
 
-@pytest.mark.parametrize("bits", ["4", "8"])
+@pytest.mark.parametrize("bits", [4, 8])
 @pytest.mark.parametrize("parents", ["any", "min_id"])
-def test_level_mirror_widths(tq, monkeypatch, bits, parents):
+def test_level_mirror_widths(tq, bits, parents):
     """Both level-mirror widths (R8; the plan picks nibbles above
-    2^25 vertices, TQ_MIRROR_BITS forces one): identical levels on graphs
+    2^25 vertices, bfs_opts.mirror_bits forces one): identical levels on graphs
     whose depth stays below, crosses and far exceeds the nibble's saturation
     (14) and the byte's (254), with delay injection perturbing the schedule."""
-    monkeypatch.setenv("TQ_MIRROR_BITS", bits)
     graphs = [kronecker_csr(12, 16, 5), grid_csr(40, 23),
               edges_to_csr(np.arange(599), np.arange(1, 600), 600, "path600"), tree4_csr(20000)]
     for g in graphs:
         rp, col = to_dev(g)
         roots = [0, int(sample_roots(g.row_ptr, 1, seed=9)[0])]
-        with tq.BfsPlan(rp, col, parents=parents, timeout_s=20) as plan:
+        with tq.BfsPlan(rp, col, parents=parents, timeout_s=20, mirror_bits=bits) as plan:
             import torch
             lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
             pa = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
@@ -398,7 +397,7 @@ def test_level_mirror_widths(tq, monkeypatch, bits, parents):
                 st = plan.run(root, lv, pa)
                 check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
         with tq.BfsPlan(rp, col, parents=parents, timeout_s=20, debug_delay_ns=2000,
-                        debug_delay_seed=3) as plan:
+                        debug_delay_seed=3, mirror_bits=bits) as plan:
             st = plan.run(roots[1], lv, pa)
             check_against_oracle(g, roots[1], lv, pa, st, min_id=parents == "min_id")
 
@@ -429,3 +428,41 @@ def test_deep_graph_plans_shrink_the_grid(tq):
     with tq.BfsPlan(rp, col) as plan:
         plan.run(int(sample_roots(g.row_ptr, 1, 1)[0]), lv, None)
         assert plan.run(int(sample_roots(g.row_ptr, 1, 2)[0]), lv, None)["persistent_threads"] == full
+
+
+@pytest.mark.parametrize("t_main,t_chunk", [((1 << 32) - 3000, (1 << 32) - 40),
+                                            (5 * (1 << 32) - 1, (1 << 33) - 1),
+                                            ((1 << 61) + (1 << 32) - 2000, (1 << 32) - 7)])
+@pytest.mark.parametrize("parents", ["any", "min_id"])
+def test_runs_across_the_32bit_ticket_wrap(tq, t_main, t_chunk, parents):
+    """The kernel keeps the low 32 bits of a ticket (slot and sequence tag,
+    DESIGN.md R1); a plan that has run many BFS carries its tickets on across
+    runs (bench.py: ~1,600 scale-26 runs reach ~5e10 tickets, crossing 2^32
+    about ten times).  Start both queues just below a 2^32 multiple
+    (bfs_plan_set_tickets) and check levels and parents of consecutive runs on
+    both sides of the wrap, with hub chunks (chunk = 32) in the chunk queue."""
+    import torch
+    g = kronecker_csr(12, 16, 3)
+    rp, col = to_dev(g)
+    lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+    pa = torch.empty_like(lv)
+    roots = [int(r) for r in sample_roots(g.row_ptr, 4, 21)]
+    with tq.BfsPlan(rp, col, chunk=32, parents=parents, timeout_s=20) as plan:
+        plan.set_tickets(t_main, t_chunk)
+        assert plan.tickets() == (t_main, t_chunk)
+        for r in roots:
+            st = plan.run(r, lv, pa)
+            check_against_oracle(g, r, lv, pa, st, min_id=parents == "min_id")
+        m, c = plan.tickets()
+        assert m > t_main and c > t_chunk
+        assert (m >> 32) > (t_main >> 32) and (c >> 32) > (t_chunk >> 32)  # both crossed a 2^32 multiple
+
+
+def test_set_tickets_argument_checks(tq):
+    g = kronecker_csr(8, 16, 1)
+    rp, col = to_dev(g)
+    with tq.BfsPlan(rp, col) as plan:
+        with pytest.raises(tq.TQError):
+            plan.set_tickets(1 << 62, 0)
+        with pytest.raises(tq.TQError):
+            plan.set_tickets(0, 1 << 63)

@@ -36,6 +36,9 @@ def test_grid4096_closed_form(tq):
         assert torch.equal(level.long(), r + c)
         lp = level.long()[parent.long()]
         assert torch.equal(lp[1:], level.long()[1:] - 1) and int(parent[0]) == 0
+        # Graph500 rules (tree edges are CSR edges, no edge spans > 1 level)
+        assert oracle.validate_tree(rp.cpu().numpy(), col.cpu().numpy(), 0, level.cpu().numpy(),
+                                    parent.cpu().numpy()) == (0, -1)
         if parents == "min_id":
             exp = torch.where(r > 0, v - rows, v - 1)
             exp[0] = 0
@@ -43,7 +46,7 @@ def test_grid4096_closed_form(tq):
         assert st["traversed_edges"] == 2 * rows * (rows - 1) and st["max_level"] == 2 * rows - 2
 
 
-def _kron_check(tq, scale, n_roots):
+def _kron_check(tq, scale, n_roots, t0=None):
     import torch
     import inputs.gpu as gg
     from inputs import sample_roots
@@ -53,6 +56,8 @@ def _kron_check(tq, scale, n_roots):
     level = torch.empty(n, dtype=torch.int32, device="cuda")
     parent = torch.empty_like(level)
     with tq.BfsPlan(rp, col) as plan:
+        if t0 is not None:  # start the queues just below a 2^32 wrap of the sequence tags
+            plan.set_tickets(*t0)
         for root in sample_roots(rp_h, n_roots, 2):
             st = plan.run(int(root), level, parent)
             lv_o, _, info = oracle.bfs(rp_h, col_h, int(root), parents=False)
@@ -62,12 +67,20 @@ def _kron_check(tq, scale, n_roots):
             pa = parent.cpu().numpy()
             reached = lv_o > 0
             assert np.all(lv_o[pa[reached]] == lv_o[reached] - 1)
+            # the default parent rule ('any') at full size: every Graph500 rule,
+            # including that each tree edge (parent[v], v) is a CSR edge
+            assert oracle.validate_tree(rp_h, col_h, int(root), lv, pa) == (0, -1)
             assert st["traversed_edges"] == info["traversed_edges"]
             assert st["reached"] == info["reached"]
 
 
 def test_kron24_levels_identical(tq):
     _kron_check(tq, 24, 2)
+
+
+def test_kron24_across_the_ticket_wrap(tq):
+    # the bench's long-running plan crosses 2^32 tickets many times
+    _kron_check(tq, 24, 2, t0=((1 << 32) - 5_000_000, (1 << 32) - 3_000))
 
 
 def test_kron26_levels_identical(tq):

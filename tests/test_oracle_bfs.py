@@ -189,6 +189,42 @@ def test_validator_rejects_mutations():
     assert oracle.validate_tree(g.row_ptr, g.col, root, lv, parent)[0] == 2
 
 
+def test_validator_rule5_exactly():
+    """Rule 5 (every CSR edge spans <= 1 level, and never joins a reached and
+    an unreached vertex) must fire on inputs that satisfy rules 1-4."""
+    # path 0-1-2-3 plus chord 0-3: the path tree with levels 0,1,2,3 passes
+    # rules 1-4 (every tree edge is an edge, levels step by one) but the chord
+    # spans 3 levels -- true levels are 0,1,2,1
+    g = edges_to_csr(np.array([0, 1, 2, 0]), np.array([1, 2, 3, 3]), 4)
+    level = np.array([0, 1, 2, 3], dtype=np.int32)
+    parent = np.array([0, 0, 1, 2], dtype=np.int32)
+    assert oracle.validate_tree(g.row_ptr, g.col, 0, level, parent)[0] == 5
+    level2, parent2, _ = oracle.bfs(g.row_ptr, g.col, 0)
+    assert level2.tolist() == [0, 1, 2, 1]
+    assert oracle.validate_tree(g.row_ptr, g.col, 0, level2, parent2) == (0, -1)
+    # an edge spanning exactly 2 levels: 0-1, 1-2, 0-2 with levels 0,1,2
+    g = edges_to_csr(np.array([0, 1, 0]), np.array([1, 2, 2]), 3)
+    assert oracle.validate_tree(g.row_ptr, g.col, 0, np.array([0, 1, 2], np.int32),
+                                np.array([0, 0, 1], np.int32))[0] == 5
+    # a reached vertex with an unreached neighbour whose own fields are
+    # consistent (level -1, parent -1): path 0-1-2 cut after 1
+    g = edges_to_csr(np.array([0, 1]), np.array([1, 2]), 3)
+    rule, bad = oracle.validate_tree(g.row_ptr, g.col, 0, np.array([0, 1, -1], np.int32),
+                                     np.array([0, 0, -1], np.int32))
+    assert rule == 5 and bad in (1, 2)
+    # on a Kronecker graph: drop a whole leaf (a reached vertex whose only
+    # reached neighbours are one level up, so nobody names it as a parent)
+    gk = kronecker_csr(10, 16, 1)
+    root = int(np.argmax(gk.degrees()))
+    lv, pa, _ = oracle.bfs(gk.row_ptr, gk.col, root)
+    children = np.zeros(gk.n_vertices, dtype=bool)
+    children[pa[(pa >= 0) & (np.arange(gk.n_vertices) != root)]] = True
+    leaf = int(np.flatnonzero((lv > 0) & ~children)[0])
+    lv2, pa2 = lv.copy(), pa.copy()
+    lv2[leaf], pa2[leaf] = -1, -1
+    assert oracle.validate_tree(gk.row_ptr, gk.col, root, lv2, pa2)[0] == 5
+
+
 def test_min_id_parent_is_min_over_candidates():
     # a diamond: 0-1, 0-2, 1-3, 2-3 ; root 0 -> parent(3) = 1 (not 2)
     g = edges_to_csr(np.array([0, 0, 1, 2]), np.array([1, 2, 3, 3]), 4)
