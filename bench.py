@@ -147,6 +147,236 @@ def cpu_oracle_sample(row_ptr, col, roots, budget_s=20.0, check=None):
     return te_sum / sec_sum, done, sec_sum, lv0
 
 
+def _median(xs):
+    xs = sorted(xs)
+    return xs[len(xs) // 2] if xs else None
+
+
+def _mirror_bytes(n):
+    return n if n <= (1 << 25) else (n + 7) // 8 * 4  # byte / nibble mirror (R8)
+
+
+def _roofline(stats_list, hbm_peak, peak_src, probe_g=None):
+    """HBM roofline (SURVEY §8(d) algorithmic bytes / CUDA-event kernel time,
+    per launch) and the L2 random-probe roofline of the persistent kernel."""
+    runs = len(stats_list)
+    te = sum(s["traversed_edges"] for s in stats_list)
+    reached = sum(s["reached"] for s in stats_list)
+    kern_s = sum(s["ms_kernel"] for s in stats_list) * 1e-3 / runs
+    alg = algorithmic_bytes(te, reached) / runs
+    out = {"bound": "hbm", "achieved": round(alg / kern_s / 1e9, 1), "peak": hbm_peak, "unit": "GB/s",
+           "frac": round(alg / kern_s / 1e9 / hbm_peak, 4), "peak_source": peak_src,
+           "alg_bytes_per_launch": int(alg), "avg_launch_ms": round(kern_s * 1e3, 4)}
+    if probe_g:
+        scanned = sum(s["edges_scanned"] for s in stats_list) / runs
+        out["l2_probe"] = {"achieved": round(scanned / kern_s / 1e9, 1), "peak": round(probe_g, 1),
+                           "unit": "G CSR entries/s vs G random L2 probes/s",
+                           "frac": round(scanned / kern_s / 1e9 / probe_g, 4)}
+    return out
+
+
+def _cpu_info():
+    return {"nproc": os.cpu_count(), "cpu_model": cpu_model()}
+
+
+def config_rmat10(tq, dev, local, args):
+    """BASELINE.json configs[0]: R-MAT scale 10, single-root BFS, GPU us beside
+    the CPU oracle's ms (median of 20 each), every sampled root checked."""
+    import numpy as np
+    import torch
+    import oracle
+    rp, col = make_graph("kron", 10, 16, dev)
+    rp_h, col_h = rp.cpu().numpy(), col.cpu().numpy()
+    roots = pick_roots("kron", rp_h, 16)
+    n = rp.numel() - 1
+    lv = torch.empty(n, dtype=torch.int32, device=dev)
+    pa = torch.empty_like(lv)
+    out = {"workload": "rmat10", "graph": "kron 10 ef16", "n_vertices": n, "nnz": int(col.numel()),
+           "roots": len(roots)}
+    with ClockSampler(local) as clk:
+        ok_lv, ok_pa, ok_min = True, True, True
+        with tq.BfsPlan(rp, col, variant=args.variant, device=local) as plan, \
+                tq.BfsPlan(rp, col, variant=args.variant, device=local, parents="min_id") as pmin:
+            for r in roots[:3]:
+                plan.run(r, lv, pa)
+            us, te = [], 0
+            for i in range(20):
+                st = plan.run(roots[i % len(roots)], lv, pa)
+                us.append(st["ms"] * 1e3)
+                te += st["traversed_edges"]
+            for r in roots:  # parity of every sampled root (default and min-id rules)
+                plan.run(r, lv, pa)
+                lo, po, _ = oracle.bfs(rp_h, col_h, r)
+                lvh, pah = lv.cpu().numpy(), pa.cpu().numpy()
+                ok_lv &= bool(np.array_equal(lvh, lo))
+                ok_pa &= oracle.validate_tree(rp_h, col_h, r, lvh, pah)[0] == 0
+                pmin.run(r, lv, pa)
+                ok_min &= bool(np.array_equal(lv.cpu().numpy(), lo) and np.array_equal(pa.cpu().numpy(), po))
+        ms_o, te_o = [], 0
+        for i in range(20):
+            _, _, info = oracle.bfs(rp_h, col_h, roots[i % len(roots)], parents=False)
+            ms_o.append(info["seconds_levels"] * 1e3)
+            te_o += info["traversed_edges"]
+    out.update({
+        "gpu_us_median": round(_median(us), 2), "gpu_us_min": round(min(us), 2), "gpu_runs": 20,
+        "gpu_timed": "CUDA events around init + persistent kernel + unpack (bfs_stats.ms), graph L2-resident",
+        "gpu_gteps": round(te / (sum(us) * 1e-6) / 1e9, 4),
+        "cpu_baseline": dict({"kind": "oracle", "cores": 1, "ms_median": round(_median(ms_o), 3),
+                              "gteps": round(te_o / (sum(ms_o) * 1e-3) / 1e9, 4),
+                              "sample": "20 sequential BFS (levels), the same roots cycled"}, **_cpu_info()),
+        "parity": {"levels_identical": ok_lv, "parents_graph500_valid": ok_pa,
+                   "min_id_parents_identical": ok_min, "roots_checked": len(roots)},
+        "clocks": clk.summary()})
+    return out
+
+
+def config_grid(tq, dev, local, args, hbm_peak, peak_src):
+    """BASELINE.json configs[2]: 4096 x 4096 grid from the corner (8,191
+    levels): ms and us per level, median of 3 after 2 warm-up runs."""
+    import numpy as np
+    import torch
+    import oracle
+    rows = 4096
+    rp, col = make_graph("grid", rows, 0, dev)
+    n = rp.numel() - 1
+    lv = torch.empty(n, dtype=torch.int32, device=dev)
+    pa = torch.empty_like(lv)
+    out = {"workload": "grid4096", "graph": "grid 4096x4096, 4-neighbour", "n_vertices": n,
+           "nnz": int(col.numel()), "root": 0,
+           "l2": "inputs larger than L2 (CSR %.0f MB)" % (((n + 1) * 8 + col.numel() * 4) / 1e6)}
+    with ClockSampler(local) as clk:
+        with tq.BfsPlan(rp, col, variant=args.variant, device=local) as plan:
+            for _ in range(2):
+                plan.run(0, lv, pa)
+            sts = [plan.run(0, lv, pa) for _ in range(3)]
+        v = torch.arange(n, device=dev, dtype=torch.int64)
+        closed = bool(torch.equal(lv.long(), v // rows + v % rows))
+        rp_h, col_h = rp.cpu().numpy(), col.cpu().numpy()
+        rule = oracle.validate_tree(rp_h, col_h, 0, lv.cpu().numpy(), pa.cpu().numpy())[0]
+        lo, _, info = oracle.bfs(rp_h, col_h, 0, parents=False)
+    ms = _median([s["ms"] for s in sts])
+    levels = sts[0]["max_level"] + 1
+    out.update({
+        "ms_median": round(ms, 3), "ms_kernel_median": round(_median([s["ms_kernel"] for s in sts]), 3),
+        "us_per_level": round(ms * 1e3 / levels, 3), "levels": levels,
+        "gteps": round(sts[0]["traversed_edges"] / (ms * 1e-3) / 1e9, 4),
+        "persistent_threads": sts[0]["persistent_threads"],
+        "roofline": _roofline(sts, hbm_peak, peak_src),
+        "cpu_baseline": dict({"kind": "oracle", "cores": 1, "ms": round(info["seconds_levels"] * 1e3, 1),
+                              "gteps": round(info["traversed_edges"] / info["seconds_levels"] / 1e9, 4),
+                              "sample": "one sequential BFS (levels) from the corner"}, **_cpu_info()),
+        "parity": {"levels_closed_form_r_plus_c": closed, "levels_identical": bool(np.array_equal(lv.cpu().numpy(), lo)),
+                   "parents_graph500_valid": rule == 0},
+        "clocks": clk.summary()})
+    return out
+
+
+def config_kron24(tq, dev, local, args, hbm_peak, peak_src):
+    """BASELINE.json configs[3]: Kronecker scale 24 on one B200: one root
+    (median of 5 after a warm-up) and an 8-root batch, HBM and L2-probe
+    rooflines, the oracle on the first root."""
+    import numpy as np
+    import torch
+    import oracle
+    rp, col = make_graph("kron", 24, 16, dev)
+    rp_h = rp.cpu().numpy()
+    roots = pick_roots("kron", rp_h, 8)
+    n = rp.numel() - 1
+    lv = torch.empty(n, dtype=torch.int32, device=dev)
+    pa = torch.empty_like(lv)
+    out = {"workload": "kron24", "graph": "kron 24 ef16", "n_vertices": n, "nnz": int(col.numel()),
+           "roots": roots, "l2": "inputs larger than L2 (CSR %.0f MB)" % (((n + 1) * 8 + col.numel() * 4) / 1e6)}
+    with ClockSampler(local) as clk:
+        with tq.BfsPlan(rp, col, variant=args.variant, device=local) as plan:
+            plan.run(roots[1], lv, pa)
+            single = [plan.run(roots[0], lv, pa) for _ in range(5)]
+            lv0, pa0 = lv.cpu().numpy(), pa.cpu().numpy()
+            batch = [plan.run(r, lv, pa) for _ in range(2) for r in roots]
+        probe_g = tq.probe_ceiling(_mirror_bytes(n), 1 << 28, device=local)
+        col_h = col.cpu().numpy()
+        lo, _, info = oracle.bfs(rp_h, col_h, roots[0], parents=False)
+        rule = oracle.validate_tree(rp_h, col_h, roots[0], lv0, pa0)[0]
+    s0 = single[2]
+    ms1 = _median([s["ms"] for s in single])
+    out.update({
+        "single_root": {"root": roots[0], "ms_median": round(ms1, 4),
+                        "gteps": round(s0["traversed_edges"] / (ms1 * 1e-3) / 1e9, 3),
+                        "roofline": _roofline(single, hbm_peak, peak_src, probe_g)},
+        "batch8": {"gteps": round(sum(s["traversed_edges"] for s in batch) / (sum(s["ms"] for s in batch) * 1e-3) / 1e9, 3),
+                   "gteps_kernel_only": round(sum(s["traversed_edges"] for s in batch) /
+                                              (sum(s["ms_kernel"] for s in batch) * 1e-3) / 1e9, 3),
+                   "runs": len(batch), "roofline": _roofline(batch, hbm_peak, peak_src, probe_g)},
+        "cpu_baseline": dict({"kind": "oracle", "cores": 1, "ms": round(info["seconds_levels"] * 1e3, 1),
+                              "gteps": round(info["traversed_edges"] / info["seconds_levels"] / 1e9, 4),
+                              "sample": "one sequential BFS (levels) of the first root"}, **_cpu_info()),
+        "parity": {"root": roots[0], "levels_identical": bool(np.array_equal(lv0, lo)),
+                   "parents_graph500_valid": rule == 0},
+        "clocks": clk.summary()})
+    return out
+
+
+def config_queue(tq, local, args):
+    """BASELINE.json configs[1]: queue throughput and weak-scaling efficiency
+    E(P) = (X(P) / P) / (X(1 group) / 1 group) at full occupancy for the warp
+    proxy (the paper's) and the pipelined CTA proxy ("thread
+    group"), b = 1 / 8 / 32, 1,024 iterations per warp; the single-group rate
+    is the median of 5 runs of the same variant and depth.  Comparators at
+    b = 32 and the same-address atomic ceiling.  Every run's item multiset is
+    checked (count, sum and xor of splitmix64 over the items)."""
+    import numpy as np
+    import oracle
+    from inputs import fingerprint, item_of
+    iters, cap = 1024, 1 << 22
+
+    def run(v, w, b, d, items=None):
+        items = items or w * b * iters
+        r = tq.queue_bench(v, warps=w, batch=b, items=items, capacity=cap, seed=3, depth=d, device=local,
+                           timeout_s=30)
+        exp = fingerprint(item_of(3, np.arange(r["items"])))
+        ok = ((r["enq"], r["sum_enq"], r["xor_enq"]) == tuple(exp) and
+              (r["deq"], r["sum_deq"], r["xor_deq"]) == tuple(exp))
+        return r, 2 * r["items"] / (r["ms"] * 1e-3) / 1e6, ok
+
+    full_w = tq.queue_bench("rf_an", warps=0, batch=1, items=1 << 20, capacity=cap, device=local)["warps"]
+    out = {"unit": "M ops/s (enqueue + dequeue)", "capacity": cap, "iters_per_warp": iters,
+           "full_threads": 32 * full_w, "scaling": []}
+    conserved = True
+    with ClockSampler(local) as clk:
+        for v, d, g in (("rf_an", 1, 1), ("rf_an_cta", 2, 8)):
+            for b in (1, 8, 32):
+                base = []
+                for _ in range(5):
+                    _, x, ok = run(v, g, b, d)
+                    base.append(x / g)
+                    conserved &= ok
+                w_full = tq.queue_bench(v, warps=0, batch=b, items=1 << 22, capacity=cap, depth=d,
+                                        device=local)["warps"]
+                r, x, ok = run(v, w_full, b, d)
+                conserved &= ok
+                w = r["warps"]
+                out["scaling"].append({"variant": v, "depth": d, "group_warps": g, "b": b, "threads": 32 * w,
+                                       "mops": round(x, 1), "single_group_mops_per_warp": round(_median(base), 3),
+                                       "E": round(x / w / _median(base), 3),
+                                       "atomics_per_item": round(r["atomics"] / r["items"], 4)})
+        comps = []
+        for v in ("per_thread_afa", "cas_retry", "an"):
+            r, x, ok = run(v, 0, 32, 1, items=full_w * 32 * 64)
+            conserved &= ok
+            comps.append({"variant": v, "b": 32, "threads": 32 * r["warps"], "mops": round(x, 1),
+                          "atomics_per_item": round(r["atomics"] / r["items"], 4),
+                          "cas_failures_per_item": round(r["cas_failures"] / r["items"], 4)})
+        out["comparators"] = comps
+        r = tq.queue_bench("atomic_ceiling", warps=0, batch=32, items=1 << 24, capacity=cap, device=local)
+        out["same_address_atomics_per_s_G"] = round(r["atomics"] / (r["ms"] * 1e-3) / 1e9, 3)
+    n = 1 << 22
+    sec, _ = oracle.queue_replay(cap, item_of(3, np.arange(n)), 32)
+    out["cpu_baseline"] = dict({"kind": "oracle", "cores": 1, "mops": round(2 * n / sec / 1e6, 1),
+                                "sample": "sequential ticket model, 2^22 items in batches of 32"}, **_cpu_info())
+    out["conserved"] = bool(conserved)
+    out["clocks"] = clk.summary()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -159,6 +389,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-queue", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="skip configs 1-4 (headline workload only)")
     ap.add_argument("--cpu-budget", type=float, default=20.0)
     ap.add_argument("--parents", default="any", choices=["any", "min_id"])
     args = ap.parse_args()
@@ -327,30 +558,6 @@ def main():
                "timed": "host perf_counter per step around bfs_plan_create(pinned host CSR: H2D) + "
                         "bfs_plan_run_batch(all roots, pinned host level/parent: D2H per root), synchronised"}
 
-    # ---- queue throughput on this GPU (BASELINE metric's second half, config 2
-    # at full occupancy; outside the BFS timed region, device-timed by tq_bench;
-    # after the e2e leg, whose first plan would otherwise grow the memory pool) ----
-    queue = None
-    if not args.no_queue:
-        from inputs import fingerprint, item_of
-        queue = {"unit": "M ops/s (enqueue + dequeue)", "items": 1 << 24, "per_gpu": True,
-                 "capacity": 1 << 22, "runs": []}
-        for v, b, d in (("rf_an", 1, 1), ("rf_an", 32, 1), ("rf_an_cta", 32, 2), ("per_thread_afa", 32, 1),
-                        ("atomic_ceiling", 32, 1)):
-            r = tq.queue_bench(v, warps=0, batch=b, items=1 << 24, capacity=1 << 22, seed=3, depth=d,
-                               device=local, timeout_s=30)
-            rec = {"variant": v, "batch": b, "depth": d, "threads": 32 * r["warps"],
-                   "mops": round(2 * r["items"] / (r["ms"] * 1e-3) / 1e6, 1),
-                   "atomics_per_item": round(r["atomics"] / r["items"], 4)}
-            if v == "atomic_ceiling":
-                rec = {"variant": v, "threads": rec["threads"],
-                       "same_address_atomics_per_s_G": round(r["atomics"] / (r["ms"] * 1e-3) / 1e9, 3)}
-            else:
-                exp = fingerprint(item_of(3, np.arange(r["items"])))
-                rec["conserved"] = ((r["enq"], r["sum_enq"], r["xor_enq"]) == tuple(exp) and
-                                    (r["deq"], r["sum_deq"], r["xor_deq"]) == tuple(exp))
-            queue["runs"].append(rec)
-
     # ---- CPU baseline: the oracle, 1 core, bounded sample, rank 0 at N=1 ----
     cpu = None
     parity = None
@@ -370,6 +577,29 @@ def main():
                "nproc": os.cpu_count(), "cpu_model": cpu_model(),
                "sample": f"{len(done)} of the {len(roots)} roots of the same graph, sequential "
                          f"BFS levels only ({sec:.1f} s of CPU)"}
+
+    # ---- the other BASELINE.json configs on this GPU (rank 0; after the timed
+    # region and the e2e leg): config 1 (R-MAT s10, GPU us beside the oracle's
+    # ms), config 2 (queue throughput + E(P)), config 3 (grid 4096^2, us per
+    # level), config 4 (Kronecker s24, one root + 8 roots, rooflines) ----
+    configs = None
+    if rank == 0 and not args.no_configs:
+        configs = {}
+        for key, fn in (("2_queue", lambda: config_queue(tq, local, args)),
+                        ("1_rmat10", lambda: config_rmat10(tq, dev, local, args)),
+                        ("3_grid4096", lambda: config_grid(tq, dev, local, args, hbm_peak, peak_src)),
+                        ("4_kron24", lambda: config_kron24(tq, dev, local, args, hbm_peak, peak_src))):
+            if key == "2_queue" and args.no_queue:
+                continue
+            t_c = time.time()
+            try:
+                configs[key] = fn()
+            except Exception as ex:  # report, do not lose the headline line
+                configs[key] = {"error": f"{type(ex).__name__}: {ex}"}
+            configs[key]["wall_s"] = round(time.time() - t_c, 1)
+            torch.cuda.empty_cache()
+    if dist:
+        dist.barrier()
 
     csr_mb = ((n + 1) * 8 + col.numel() * 4) / 1e6
     if rank == 0:
@@ -401,7 +631,7 @@ def main():
                          "alg_bytes_per_launch": int(alg_bytes),
                          "avg_launch_ms": round(avg_kernel_s * 1e3, 4)},
             "roofline_l2_probe": probe_roof,
-            "queue": queue,
+            "configs": configs,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,
