@@ -319,19 +319,21 @@ def config_queue(tq, local, args):
     """BASELINE.json configs[1]: queue throughput and weak-scaling efficiency
     E(P) = (X(P) / P) / (X(1 group) / 1 group) at full occupancy for the warp
     proxy (the paper's) and the pipelined CTA proxy ("thread
-    group"), b = 1 / 8 / 32, 1,024 iterations per warp; the single-group rate
-    is the median of 5 runs of the same variant and depth.  Comparators at
-    b = 32 and the same-address atomic ceiling.  Every run's item multiset is
-    checked (count, sum and xor of splitmix64 over the items)."""
+    group", with acquire and with relaxed arrival checks), b = 1 / 8 / 32,
+    1,024 iterations per warp; the single-group rate is the median of 5 runs
+    of the same variant, depth and poll.  Comparators at b = 32 (CAS queues
+    naive and with a bounded back-off) and the same-address atomic ceiling.
+    Every run's item multiset is checked (count, sum and xor of splitmix64
+    over the items)."""
     import numpy as np
     import oracle
     from inputs import fingerprint, item_of
     iters, cap = 1024, 1 << 22
 
-    def run(v, w, b, d, items=None):
+    def run(v, w, b, d, items=None, relaxed=False, backoff=0):
         items = items or w * b * iters
         r = tq.queue_bench(v, warps=w, batch=b, items=items, capacity=cap, seed=3, depth=d, device=local,
-                           timeout_s=30)
+                           timeout_s=30, relaxed_poll=relaxed, cas_backoff_ns=backoff)
         exp = fingerprint(item_of(3, np.arange(r["items"])))
         ok = ((r["enq"], r["sum_enq"], r["xor_enq"]) == tuple(exp) and
               (r["deq"], r["sum_deq"], r["xor_deq"]) == tuple(exp))
@@ -342,29 +344,37 @@ def config_queue(tq, local, args):
            "full_threads": 32 * full_w, "scaling": []}
     conserved = True
     with ClockSampler(local) as clk:
-        for v, d, g in (("rf_an", 1, 1), ("rf_an_cta", 2, 8)):
+        for v, d, g, relaxed in (("rf_an", 1, 1, False), ("rf_an_cta", 2, 8, False), ("rf_an_cta", 2, 8, True)):
             for b in (1, 8, 32):
                 base = []
                 for _ in range(5):
-                    _, x, ok = run(v, g, b, d)
+                    _, x, ok = run(v, g, b, d, relaxed=relaxed)
                     base.append(x / g)
                     conserved &= ok
                 w_full = tq.queue_bench(v, warps=0, batch=b, items=1 << 22, capacity=cap, depth=d,
                                         device=local)["warps"]
-                r, x, ok = run(v, w_full, b, d)
+                r, x, ok = run(v, w_full, b, d, relaxed=relaxed)
                 conserved &= ok
                 w = r["warps"]
-                out["scaling"].append({"variant": v, "depth": d, "group_warps": g, "b": b, "threads": 32 * w,
+                out["scaling"].append({"variant": v, "depth": d, "group_warps": g, "b": b,
+                                       "poll": "relaxed" if relaxed else "acquire", "threads": 32 * w,
                                        "mops": round(x, 1), "single_group_mops_per_warp": round(_median(base), 3),
                                        "E": round(x / w / _median(base), 3),
                                        "atomics_per_item": round(r["atomics"] / r["items"], 4)})
+        # comparators at b = 32, at the paper's 14,336 threads and at
+        # full occupancy; the CAS queues naive and with a bounded back-off
         comps = []
-        for v in ("per_thread_afa", "cas_retry", "an"):
-            r, x, ok = run(v, 0, 32, 1, items=full_w * 32 * 64)
-            conserved &= ok
-            comps.append({"variant": v, "b": 32, "threads": 32 * r["warps"], "mops": round(x, 1),
-                          "atomics_per_item": round(r["atomics"] / r["items"], 4),
-                          "cas_failures_per_item": round(r["cas_failures"] / r["items"], 4)})
+        for v, bo in (("rf_an", 0), ("per_thread_afa", 0), ("cas_retry", 0), ("cas_retry", 2048), ("an", 0),
+                      ("an", 2048)):
+            for w in (448, 0):
+                it = 2 if v in ("cas_retry", "an") else 16
+                w_run = w or tq.queue_bench(v, warps=0, batch=32, items=1 << 22, capacity=cap,
+                                            device=local)["warps"]
+                r, x, ok = run(v, w_run, 32, 1, items=w_run * 32 * it, backoff=bo)
+                conserved &= ok
+                comps.append({"variant": v, "cas_backoff_ns": bo, "b": 32, "threads": 32 * r["warps"],
+                              "mops": round(x, 1), "atomics_per_item": round(r["atomics"] / r["items"], 4),
+                              "cas_failures_per_item": round(r["cas_failures"] / r["items"], 4)})
         out["comparators"] = comps
         r = tq.queue_bench("atomic_ceiling", warps=0, batch=32, items=1 << 24, capacity=cap, device=local)
         out["same_address_atomics_per_s_G"] = round(r["atomics"] / (r["ms"] * 1e-3) / 1e9, 3)

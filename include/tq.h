@@ -181,6 +181,10 @@ typedef struct {
                            == 1, so tokens are expanded late and with stale
                            levels.  0 = off (default); at most 1,000,000     */
     uint32_t debug_delay_seed;
+    int cas_backoff_ns; /* CAS_RETRY / AN only: after a failed CAS, sleep 32 ns
+                           doubling up to this many ns before retrying (a
+                           bounded exponential back-off); 0 = retry at once
+                           (the naive form); 0..1,000,000                   */
     int mirror_bits;    /* level-mirror width (R8): 0 = auto (a nibble
                            per vertex when a byte mirror would exceed 32 MB,
                            RF_AN only; else a byte), 8 = byte, 4 = nibble
@@ -318,6 +322,13 @@ typedef struct {
     int cluster;        /* RF_AN_CLUSTER: CTAs per cluster (0 = 4; 1..16);
                            warps must be a multiple of 8*cluster and fit the
                            co-resident cluster count, else TQ_ERR_INVALID    */
+    int cas_backoff_ns; /* CAS_RETRY / AN: bounded exponential back-off after
+                           a failed CAS (32 ns doubling up to this); 0 =
+                           none (the naive form); 0..1,000,000              */
+    int relaxed_poll;   /* 1: the arrival check is a relaxed load and the
+                           acquire is skipped (the benchmark's items carry
+                           their whole payload, so nothing else must become
+                           visible); 0 = acquire load per poll (tq_take)    */
 } tq_bench_cfg;
 
 typedef struct {

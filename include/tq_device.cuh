@@ -206,6 +206,22 @@ __device__ __forceinline__ bool tq_take(const tq_device_view &q, unsigned long l
     return true;
 }
 
+/* tq_take with a relaxed arrival check (ld.relaxed.gpu: served by L2, no
+ * L1 invalidation per poll).  For items that carry their whole payload: a
+ * hit makes the item visible, but NOT other data the producer wrote before
+ * publishing it -- use tq_take when the item names such data. */
+__device__ __forceinline__ bool tq_take_relaxed(const tq_device_view &q, unsigned long long ticket,
+                                                unsigned int *item)
+{
+    if (ticket == TQ_NO_TICKET) return false;
+    unsigned long long *s = q.slots + (ticket & q.mask);
+    const unsigned long long v = tq_ld_relaxed(s);
+    if ((unsigned int)v != (unsigned int)(ticket + 1)) return false;
+    *item = (unsigned int)(v >> 32);
+    tq_st_relaxed(s, (unsigned long long)(unsigned int)(ticket + q.mask + 1));
+    return true;
+}
+
 /* ---------------------------------------------------------------- */
 /* Listing 3: enqueue.                                    */
 /* tq_warp_reserve_rear: lane 0 reserves `n_warp` tickets at Rear     */

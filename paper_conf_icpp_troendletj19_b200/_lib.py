@@ -42,7 +42,7 @@ class bfs_opts(ctypes.Structure):
                 ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int),
                 ("parent_rule", ctypes.c_int), ("hub_queue", ctypes.c_int),
                 ("debug_delay_ns", ctypes.c_int), ("debug_delay_seed", c_u32),
-                ("mirror_bits", ctypes.c_int), ("deep_grid", ctypes.c_int), ("l2_persist", ctypes.c_int)]
+                ("cas_backoff_ns", ctypes.c_int), ("mirror_bits", ctypes.c_int), ("deep_grid", ctypes.c_int), ("l2_persist", ctypes.c_int)]
 
 
 class bfs_stats(ctypes.Structure):
@@ -59,7 +59,7 @@ class tq_bench_cfg(ctypes.Structure):
                 ("items", c_u64), ("capacity", c_u64), ("work_iters", ctypes.c_int), ("seed", c_u64),
                 ("log_mode", ctypes.c_int), ("enq_log", c_vp), ("deq_log", c_vp), ("stream", c_vp),
                 ("timeout_s", c_dbl), ("device", ctypes.c_int), ("depth", ctypes.c_int),
-                ("cluster", ctypes.c_int)]
+                ("cluster", ctypes.c_int), ("cas_backoff_ns", ctypes.c_int), ("relaxed_poll", ctypes.c_int)]
 
 
 class tq_bench_result(ctypes.Structure):

@@ -75,17 +75,19 @@ def _csr(row_ptr, col) -> _lib.tq_csr:
 
 def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None, timeout_s=0.0,
           backoff_ns=0, device=0, parents="any", hub_queue=True, debug_delay_ns=0,
-          debug_delay_seed=0, mirror_bits=0, deep_grid=True, l2_persist=True) -> _lib.bfs_opts:
+          debug_delay_seed=0, cas_backoff_ns=0, mirror_bits=0, deep_grid=True,
+          l2_persist=True) -> _lib.bfs_opts:
     return _lib.bfs_opts(int(capacity), int(threads), int(block), int(chunk), _variant(variant),
                          stream, float(timeout_s), int(backoff_ns), int(device),
                          _lib.PARENT_RULES[parents] if isinstance(parents, str) else int(parents),
                          0 if hub_queue else -1, int(debug_delay_ns), int(debug_delay_seed) & 0xFFFFFFFF,
-                         int(mirror_bits), 0 if deep_grid else -1, 0 if l2_persist else -1)
+                         int(cas_backoff_ns), int(mirror_bits), 0 if deep_grid else -1,
+                         0 if l2_persist else -1)
 
 
 # bfs / BfsPlan keyword options that map one to one onto bfs_opts fields
 _OPT_KEYS = ("variant", "capacity", "threads", "chunk", "timeout_s", "backoff_ns", "parents", "hub_queue",
-             "debug_delay_ns", "debug_delay_seed", "mirror_bits", "deep_grid", "l2_persist")
+             "debug_delay_ns", "debug_delay_seed", "cas_backoff_ns", "mirror_bits", "deep_grid", "l2_persist")
 
 
 def _stats_dict(st: _lib.bfs_stats) -> dict:
@@ -107,7 +109,7 @@ def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool =
     (staged to the device by the library). Outputs default to the graph's
     kind of memory. `opts`: the bfs_opts fields (variant, capacity, threads,
     chunk, timeout_s, backoff_ns, parents, hub_queue, debug_delay_ns,
-    debug_delay_seed, mirror_bits, deep_grid, l2_persist).
+    debug_delay_seed, cas_backoff_ns, mirror_bits, deep_grid, l2_persist).
     """
     bad = set(opts) - set(_OPT_KEYS)
     if bad:
@@ -344,7 +346,7 @@ class Queue:
 def queue_bench(variant="rf_an", *, warps: int = 0, batch: int = 32, items: int = 1 << 24,
                 capacity: int = 1 << 20, work_iters: int = 0, seed: int = 3, log: bool = False,
                 stream=None, timeout_s: float = 0.0, device: int = 0, depth: int = 1,
-                cluster: int = 0) -> dict:
+                cluster: int = 0, cas_backoff_ns: int = 0, relaxed_poll: bool = False) -> dict:
     """`tq_bench`: enqueue/dequeue throughput of one queue variant.
 
     depth=2 pipelines one iteration ahead (rf_an, rf_an_cta; rf_an_cluster
@@ -358,7 +360,8 @@ def queue_bench(variant="rf_an", *, warps: int = 0, batch: int = 32, items: int 
         deq_log = torch.zeros(items, dtype=torch.int32, device=f"cuda:{device}")
     cfg = _lib.tq_bench_cfg(_variant(variant), int(warps), int(batch), int(items), int(capacity),
                             int(work_iters), int(seed), int(log), _ptr(enq_log), _ptr(deq_log),
-                            _stream_ptr(stream), float(timeout_s), int(device), int(depth), int(cluster))
+                            _stream_ptr(stream), float(timeout_s), int(device), int(depth), int(cluster),
+                            int(cas_backoff_ns), int(bool(relaxed_poll)))
     res = _lib.tq_bench_result()
     status = lib().tq_bench(ctypes.byref(cfg), ctypes.byref(res))
     out = {f: getattr(res, f) for f, _ in res._fields_}

@@ -303,6 +303,7 @@ struct bfs_plan {
     unsigned long long next_ticket = 0;
     bool dirty = false;
     int32_t *out_scratch = nullptr;           // for host outputs
+    int cas_backoff_ns = 0;                   // CAS variants: bounded back-off (bfs_opts)
     int delay_ns = 0;                         // test only (bfs_opts.debug_delay_ns)
     uint32_t delay_seed = 0;
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -537,6 +538,11 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         delete p;
         return TQ_ERR_INVALID;
     }
+    if (o.cas_backoff_ns < 0 || o.cas_backoff_ns > 1000000) {
+        delete p;
+        return TQ_ERR_INVALID;
+    }
+    p->cas_backoff_ns = o.cas_backoff_ns;
     p->delay_ns = o.debug_delay_ns;
     p->delay_seed = o.debug_delay_seed;
     p->task = task;
@@ -711,6 +717,7 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.timeout_ns = (unsigned long long)(p->timeout_s * 1e9);
     bp.l2_window_bytes = p->l2_window;
     bp.delay_ns = (unsigned)p->delay_ns;
+    bp.cas_backoff_ns = (unsigned)p->cas_backoff_ns;
     bp.delay_seed = p->delay_seed;
     // every slot of [t0, t0 + C) holds "empty for t" when a run starts (after
     // a reset, or at Rear after a finished run; see plan_finish)
@@ -990,6 +997,7 @@ tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
     if (c->variant < TQ_VARIANT_RF_AN || c->variant > TQ_VARIANT_RF_AN_CLUSTER) return TQ_ERR_UNSUPPORTED;
     if (c->batch < 1 || c->batch > 32 || c->items == 0 || c->warps < 0) return TQ_ERR_INVALID;
     if (c->depth < 0 || c->depth > 2) return TQ_ERR_INVALID;
+    if (c->cas_backoff_ns < 0 || c->cas_backoff_ns > 1000000) return TQ_ERR_INVALID;
     const bool cluster_v = c->variant == TQ_VARIANT_RF_AN_CLUSTER;
     const int depth = cluster_v ? 2 : (c->depth == 0 ? 1 : c->depth);
     if (depth == 2 && c->variant != TQ_VARIANT_RF_AN_CTA && !cluster_v) return TQ_ERR_UNSUPPORTED;
@@ -1049,6 +1057,8 @@ tq_status tq_bench(const tq_bench_cfg *c, tq_bench_result *r)
     bp.deq_log = c->log_mode ? c->deq_log : nullptr;
     bp.out = out;
     bp.timeout_ns = (unsigned long long)((c->timeout_s > 0 ? c->timeout_s : 60.0) * 1e9);
+    bp.cas_backoff_ns = (unsigned)c->cas_backoff_ns;
+    bp.relaxed_poll = c->relaxed_poll ? 1 : 0;
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess) e = cudaEventRecord(e0, s);
     if (e == cudaSuccess) {

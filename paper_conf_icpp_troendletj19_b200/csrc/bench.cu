@@ -43,10 +43,21 @@ __device__ __forceinline__ bool bench_publish(const tq_device_view &q, unsigned 
     return tq_publish(q, t, item);
 }
 
+// Bounded exponential back-off after a failed CAS (tq_bench_cfg.cas_backoff_ns;
+// 0 = retry at once, the naive form): 32 ns doubling up to bo_max.
+__device__ __forceinline__ void b_backoff(unsigned *bo, unsigned bo_max)
+{
+    if (!bo_max) return;
+    *bo = *bo ? min(*bo * 2, bo_max) : min(32u, bo_max);
+    __nanosleep(*bo);
+}
+
 // BASE enqueue / dequeue with the ticket returned (for the logs)
 __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t item,
-                                              unsigned long long *t_out, unsigned *atom, unsigned *fail)
+                                              unsigned long long *t_out, unsigned *atom, unsigned *fail,
+                                              unsigned bo_max)
 {
+    unsigned bo = 0;
     for (unsigned tries = 0; tries < (1u << 24); ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.rear);
         unsigned long long *s = q.slots + (pos & q.mask);
@@ -60,6 +71,7 @@ __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t 
                 return true;
             }
             ++*fail;
+            b_backoff(&bo, bo_max);
         } else if (dif < 0) {
             tq_status_set_thread(q, TQ_ABORTED_FULL);
             return false;
@@ -70,8 +82,10 @@ __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t 
 }
 
 __device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *item,
-                                             unsigned long long *t_out, unsigned *atom, unsigned *fail)
+                                             unsigned long long *t_out, unsigned *atom, unsigned *fail,
+                                             unsigned bo_max)
 {
+    unsigned bo = 0;
     for (unsigned tries = 0; tries < (1u << 12); ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.front);
         unsigned long long *s = q.slots + (pos & q.mask);
@@ -86,6 +100,7 @@ __device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *
                 return 1;
             }
             ++*fail;
+            b_backoff(&bo, bo_max);
         } else if (dif < 0) {
             return 0;
         }
@@ -152,7 +167,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                 unsigned spins = 0;
                 bool have = false;
                 while (!have) {
-                    have = tq_take(q, dt, &got_item);
+                    have = p.relaxed_poll ? tq_take_relaxed(q, dt, &got_item) : tq_take(q, dt, &got_item);
                     if (!have && (++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {
                         stop = true;
                         break;
@@ -198,10 +213,10 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                     eok = bench_publish(q, et, item);
                 }
             } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
-                if (active) eok = b_cas_enqueue(q, item, &et, &atom, &fail);
+                if (active) eok = b_cas_enqueue(q, item, &et, &atom, &fail, p.cas_backoff_ns);
             } else {  // AN: proxy CAS loop reserving `batch` slots
                 unsigned long long base = 0;
-                unsigned spins = 0;
+                unsigned spins = 0, bo = 0;
                 for (;;) {
                     if ((++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {
                         eok = false;
@@ -230,6 +245,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                         base = pos;
                         break;
                     }
+                    b_backoff(&bo, p.cas_backoff_ns);
                 }
                 et = base + lane;
                 if (active && eok) tq_st_relaxed(q.slots + (et & q.mask),
@@ -257,7 +273,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                 }
                 unsigned spins = 0;
                 while (!have) {
-                    have = tq_take(q, dt, &got_item);
+                    have = p.relaxed_poll ? tq_take_relaxed(q, dt, &got_item) : tq_take(q, dt, &got_item);
                     if (!have) {
                         ++empty;
                         if ((++spins & 1023) == 0 &&
@@ -270,7 +286,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
             } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
                 unsigned spins = 0;
                 while (!have) {
-                    have = b_cas_dequeue(q, &got_item, &dt, &atom, &fail);
+                    have = b_cas_dequeue(q, &got_item, &dt, &atom, &fail, p.cas_backoff_ns);
                     if (!have) {
                         ++empty;
                         if ((++spins & 1023) == 0 &&
@@ -281,7 +297,7 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                     }
                 }
             } else {  // AN: the proxy reserves up to n ready slots per CAS
-                unsigned spins = 0;
+                unsigned spins = 0, bo = 0;
                 for (;;) {
                     const bool need = !have;
                     const unsigned m = __ballot_sync(TQ_FULL_MASK, need);
@@ -310,7 +326,10 @@ __global__ void __launch_bounds__(256) bench_kernel(const BenchParams p)
                         if (old != pos) ++fail;
                     }
                     old = tq_shfl64(old, 0);
-                    if (old != pos) continue;
+                    if (old != pos) {
+                        b_backoff(&bo, p.cas_backoff_ns);
+                        continue;
+                    }
                     const unsigned rank = __popc(m & tq_lanemask_lt());
                     if (need && rank < k) {
                         dt = pos + rank;
@@ -508,7 +527,7 @@ __global__ void __launch_bounds__(256) bench_pipe_kernel(const BenchParams p)
             unsigned spins = 0;
             bool have = false;
             while (!have) {
-                have = tq_take(q, dt, &got_item);
+                have = p.relaxed_poll ? tq_take_relaxed(q, dt, &got_item) : tq_take(q, dt, &got_item);
                 if (!have) {
                     ++empty;
                     if ((++spins & 1023) == 0 && should_stop(q, (unsigned)warp_gid, deadline)) {

@@ -177,11 +177,21 @@ __device__ __forceinline__ T warp_sum(T x)
 // CAS-based comparison queues (BASE and AN)
 // ---------------------------------------------------------------------------
 
+// Bounded exponential back-off after a failed CAS (bfs_opts.cas_backoff_ns;
+// 0 = retry at once, the naive form): 32 ns doubling up to bo_max.
+__device__ __forceinline__ void cas_backoff(unsigned *bo, unsigned bo_max)
+{
+    if (!bo_max) return;
+    *bo = *bo ? min(*bo * 2, bo_max) : min(32u, bo_max);
+    __nanosleep(*bo);
+}
+
 // BASE dequeue of one item by one lane: a classic bounded CAS queue (per-slot
 // sequence numbers); retries on CAS failure, returns false on empty.
 __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_t *item,
-                                                unsigned *atom, unsigned *fail)
+                                                unsigned *atom, unsigned *fail, unsigned bo_max)
 {
+    unsigned bo = 0;
     for (unsigned tries = 0; tries < kMaxDeqRetries; ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.front);
         unsigned long long *s = q.slots + (pos & q.mask);
@@ -195,6 +205,7 @@ __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_
                 return true;
             }
             ++*fail;
+            cas_backoff(&bo, bo_max);
         } else if (dif < 0) {
             return false;  // queue empty: the exception BASE retries on
         }
@@ -204,8 +215,9 @@ __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_
 
 // BASE enqueue of one item by one lane; queue-full aborts (no retry).
 __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_t item,
-                                                unsigned *atom, unsigned *fail)
+                                                unsigned *atom, unsigned *fail, unsigned bo_max)
 {
+    unsigned bo = 0;
     for (unsigned tries = 0; tries < kMaxEnqRetries; ++tries) {
         const unsigned long long pos = tq_ld_relaxed(q.rear);
         unsigned long long *s = q.slots + (pos & q.mask);
@@ -218,6 +230,7 @@ __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_
                 return true;
             }
             ++*fail;
+            cas_backoff(&bo, bo_max);
         } else if (dif < 0) {
             tq_status_set_thread(q, TQ_ABORTED_FULL);
             return false;
@@ -232,10 +245,10 @@ __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_
 // item count k taken for the warp; hungry lane of rank r < k gets ticket base+r.
 __device__ __forceinline__ unsigned an_dequeue(const tq_device_view &q, unsigned n,
                                                unsigned long long *base_out, unsigned *atom,
-                                               unsigned *fail)
+                                               unsigned *fail, unsigned bo_max)
 {
     const unsigned lane = tq_lane();
-    unsigned tries = 0;
+    unsigned tries = 0, bo = 0;
     for (;;) {
         unsigned long long pos = 0;
         if (lane == 0) pos = tq_ld_relaxed(q.front);
@@ -265,6 +278,7 @@ __device__ __forceinline__ unsigned an_dequeue(const tq_device_view &q, unsigned
             *base_out = pos;
             return k;
         }
+        cas_backoff(&bo, bo_max);
         if (++tries >= kMaxDeqRetries) return 0;
     }
 }
@@ -273,9 +287,10 @@ __device__ __forceinline__ unsigned an_dequeue(const tq_device_view &q, unsigned
 // they are all empty; retries on CAS failure; aborts on queue-full.
 __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigned n,
                                                 unsigned long long *base_out, unsigned *atom,
-                                                unsigned *fail)
+                                                unsigned *fail, unsigned bo_max)
 {
     const unsigned lane = tq_lane();
+    unsigned bo = 0;
     for (unsigned tries = 0;; ++tries) {
         if (tries >= kMaxEnqRetries) {
             if (lane == 0) tq_status_set_thread(q, TQ_ABORTED_TIMEOUT);
@@ -307,6 +322,7 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
             *base_out = pos;
             return true;
         }
+        cas_backoff(&bo, bo_max);
     }
 }
 
@@ -322,7 +338,7 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const uint32_t *items,
                                                unsigned cnt, unsigned lane, unsigned *qatom,
-                                               unsigned *casfail, unsigned long long lap_end)
+                                               unsigned *casfail, unsigned long long lap_end, unsigned bo_max)
 {
     if (cnt == 0) return;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
@@ -330,7 +346,7 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
         if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
             base = tq_warp_reserve_rear(q, cnt, qatom);
         } else {
-            if (!an_reserve_rear(q, cnt, &base, qatom, casfail)) return;
+            if (!an_reserve_rear(q, cnt, &base, qatom, casfail, bo_max)) return;
         }
         // release: the W updates (and this warp's Rear reservation) are
         // ordered before the tokens that name them
@@ -376,7 +392,7 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
     } else {  // CAS_RETRY: one CAS-reserved slot per item, per lane
         tq_fence_release();
         for (unsigned i = lane; i < cnt; i += 32)
-            if (!cas_enqueue_one(q, items[i], qatom, casfail)) break;
+            if (!cas_enqueue_one(q, items[i], qatom, casfail, bo_max)) break;
     }
 }
 
@@ -384,18 +400,18 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t first, unsigned n,
                                                unsigned lane, unsigned *qatom, unsigned *casfail,
-                                               unsigned long long lap_end)
+                                               unsigned long long lap_end, unsigned bo_max)
 {
     if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
         for (unsigned i = lane; i < n; i += 32)
-            if (!cas_enqueue_one(q, CHUNK_FLAG | (first + i), qatom, casfail)) break;
+            if (!cas_enqueue_one(q, CHUNK_FLAG | (first + i), qatom, casfail, bo_max)) break;
         return;
     } else {
         unsigned long long base;
         if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
             base = tq_warp_reserve_rear(q, n, qatom);
         } else if constexpr (VARIANT == TQ_VARIANT_AN) {
-            if (!an_reserve_rear(q, n, &base, qatom, casfail)) return;
+            if (!an_reserve_rear(q, n, &base, qatom, casfail, bo_max)) return;
         }
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
             // release: a chunk token names the hub's W entry (its level), and
@@ -530,10 +546,10 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             got = !got1 && have && (unsigned)sv0 == tk + 1u;
             item = (uint32_t)((got1 ? sv1 : sv0) >> 32);
         } else if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
-            got = cas_dequeue_one(q, &item, &st_qatom, &st_fail);
+            got = cas_dequeue_one(q, &item, &st_qatom, &st_fail, p.cas_backoff_ns);
         } else {  // AN: every lane is hungry each cycle (no held tickets)
             unsigned long long base = 0;
-            const unsigned k = an_dequeue(q, 32, &base, &st_qatom, &st_fail);
+            const unsigned k = an_dequeue(q, 32, &base, &st_qatom, &st_fail, p.cas_backoff_ns);
             if (lane < k) {
                 unsigned long long *s = q.slots + ((base + lane) & q.mask);
                 const unsigned long long v = tq_ld_relaxed(s);
@@ -886,7 +902,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
             if (cnt > kStageCap - 32 * KU) {
                 __syncwarp();
-                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end);
+                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end, p.cas_backoff_ns);
                 __syncwarp();
                 cnt = 0;
             }
@@ -894,7 +910,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
-        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end);
+        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end, p.cas_backoff_ns);
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
         while (hubm) {
@@ -903,7 +919,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             const unsigned n = __shfl_sync(TQ_FULL_MASK, nch, h);
             const uint32_t first = __shfl_sync(TQ_FULL_MASK, chb, h);
             enqueue_chunks<VARIANT>(hubq ? q1 : q, first, n, lane, &st_qatom, &st_fail,
-                                    hubq ? p.q1_lap_end : p.q_lap_end);
+                                    hubq ? p.q1_lap_end : p.q_lap_end, p.cas_backoff_ns);
         }
 
         // ---- completion accounting for WorkRemains() (R6) ----

@@ -96,6 +96,7 @@ struct BfsParams {
     // (t0 + C of each queue), so their enqueue skips the full check
     unsigned long long q_lap_end;
     unsigned long long q1_lap_end;
+    unsigned cas_backoff_ns;   // CAS variants: max back-off after a failed CAS (0 = none)
 };
 
 // bfs.cu
@@ -120,6 +121,8 @@ struct BenchParams {
     uint32_t *deq_log;
     unsigned long long *out;   // [0..] counters (see bench.cu)
     unsigned long long timeout_ns;
+    unsigned cas_backoff_ns;   // CAS variants: max back-off after a failed CAS (0 = none)
+    int relaxed_poll;          // 1: relaxed arrival checks (tq_take_relaxed)
 };
 cudaError_t launch_bench(int variant, const BenchParams &p, int blocks, int block, cudaStream_t s);
 cudaError_t bench_occupancy(int variant, int block, int *blocks_per_sm);
