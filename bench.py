@@ -34,6 +34,7 @@ WORKLOADS = {
     "kron24x8": ("kron", 24, 16, 8),
     "grid4096": ("grid", 4096, 0, 1),
     "rmat10": ("kron", 10, 16, 16),
+    "kron20x16": ("kron", 20, 16, 16),  # tests: a quick multi-root batch
 }
 GRAPH_SEED, ROOT_SEED = 1, 2
 
@@ -94,6 +95,15 @@ class ClockSampler:
         s = sorted(self.samples)
         return {"sm_mhz": s[len(s) // 2] if s else None, "sm_max_mhz": self.max_mhz,
                 "reasons": sorted(self.reasons), "samples": len(s)}
+
+
+def free_port():
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
 
 
 def cpu_model():
@@ -346,10 +356,11 @@ def config_queue(tq, local, args):
     with ClockSampler(local) as clk:
         for v, d, g, relaxed in (("rf_an", 1, 1, False), ("rf_an_cta", 2, 8, False), ("rf_an_cta", 2, 8, True)):
             for b in (1, 8, 32):
-                base = []
+                base, base_empty = [], []
                 for _ in range(5):
-                    _, x, ok = run(v, g, b, d, relaxed=relaxed)
+                    r1, x, ok = run(v, g, b, d, relaxed=relaxed)
                     base.append(x / g)
+                    base_empty.append(r1["empty_retries"] / r1["items"])
                     conserved &= ok
                 w_full = tq.queue_bench(v, warps=0, batch=b, items=1 << 22, capacity=cap, depth=d,
                                         device=local)["warps"]
@@ -360,6 +371,10 @@ def config_queue(tq, local, args):
                                        "poll": "relaxed" if relaxed else "acquire", "threads": 32 * w,
                                        "mops": round(x, 1), "single_group_mops_per_warp": round(_median(base), 3),
                                        "E": round(x / w / _median(base), 3),
+                                       "us_per_iteration": round(2 * b / (x / w), 3),
+                                       "single_group_us_per_iteration": round(2 * b / _median(base), 3),
+                                       "empty_polls_per_item": round(r["empty_retries"] / r["items"], 3),
+                                       "single_group_empty_polls_per_item": round(_median(base_empty), 3),
                                        "atomics_per_item": round(r["atomics"] / r["items"], 4)})
         # comparators at b = 32, at the paper's 14,336 threads and at
         # full occupancy; the CAS queues naive and with a bounded back-off
@@ -427,13 +442,17 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     coll_dev = dev if backend == "nccl" else None  # device of the collectives' tensors
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
-        if backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
-        else:
-            dist.init_process_group(backend)
+    # The process group is created at every N, N = 1 included (a one-rank NCCL
+    # group on a plain `python bench.py`), so the N > 1 code path -- barriers
+    # and the NCCL all-gather of per-rank stats -- runs in every bench run.
+    import torch.distributed as dist
+    if "MASTER_ADDR" not in os.environ:  # plain launch: a one-rank rendezvous on loopback
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ.setdefault("MASTER_PORT", str(free_port()))
+    if backend == "nccl":
+        dist.init_process_group("nccl", device_id=dev, rank=rank, world_size=world)
+    else:
+        dist.init_process_group(backend, rank=rank, world_size=world)
 
     import paper_conf_icpp_troendletj19_b200 as tq
     from paper_conf_icpp_troendletj19_b200 import multiroot
@@ -536,20 +555,45 @@ def main():
         if dist:
             dist.barrier()
         torch.cuda.synchronize(dev)
+        # Step k+1's plan (its 9 GB H2D of the pinned host CSR, in 32 MiB
+        # pieces on its own stream) is built by a helper thread while step k's
+        # batch runs: every step's H2D and D2H stay inside the timed region,
+        # overlapped with the BFS of the neighbouring step (ctypes releases the
+        # GIL during the C calls).
+        streams = [stream, torch.cuda.Stream(dev)]
+
+        def make_plan(k):
+            return tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[k % 2], device=local,
+                              parents=args.parents)
+
         t0 = time.perf_counter()
         te_e2e = 0
         step_s = []
-        for _ in range(args.steps):
+        nxt = make_plan(0)
+        for k in range(args.steps):
             ts0 = time.perf_counter()
-            with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=stream, device=local,
-                            parents=args.parents) as hp:
-                ts1 = time.perf_counter()  # bfs_plan_create returns after the H2D copies
-                # one C-ABI call per step: every root's level and parent arrays
-                # are copied to the (reused) pinned host buffers, D2H overlapped
-                # with the next root's BFS on a second stream
-                for s in hp.run_batch(mine, lv_np, pa_np, stride=0):
-                    te_e2e += s["traversed_edges"]
-                ts2 = time.perf_counter()
+            hp, box, th = nxt, {}, None
+            if k + 1 < args.steps:
+                def build(k=k, box=box):
+                    try:
+                        box["plan"] = make_plan(k + 1)
+                    except Exception as ex:  # re-raised in the main thread
+                        box["error"] = ex
+                th = threading.Thread(target=build)
+                th.start()
+            # one C-ABI call per step: every root's level and parent arrays
+            # are copied to the (reused) pinned host buffers, D2H overlapped
+            # with the next root's BFS on a second stream
+            for s_ in hp.run_batch(mine, lv_np, pa_np, stride=0):
+                te_e2e += s_["traversed_edges"]
+            ts1 = time.perf_counter()
+            if th is not None:
+                th.join()
+                if "error" in box:
+                    raise box["error"]
+                nxt = box["plan"]
+            ts2 = time.perf_counter()
+            hp.close()
             step_s.append([round(ts1 - ts0, 3), round(ts2 - ts1, 3), round(time.perf_counter() - ts2, 3)])
         torch.cuda.synchronize(dev)
         sec = time.perf_counter() - t0
@@ -564,9 +608,11 @@ def main():
         e2e = {"value": te_tot / sec_max / 1e9, "unit": "GTEPS",
                "h2d_bytes_per_step": int((n + 1) * 8 + col.numel() * 4),
                "d2h_bytes_per_step": int(len(mine) * n * 8),
-               "step_s_create_batch_destroy": step_s,
-               "timed": "host perf_counter per step around bfs_plan_create(pinned host CSR: H2D) + "
-                        "bfs_plan_run_batch(all roots, pinned host level/parent: D2H per root), synchronised"}
+               "step_s_batch_wait_destroy": step_s,
+               "timed": "host perf_counter from the first bfs_plan_create (pinned host CSR: H2D) to the "
+                        "last step's synchronised end; per step bfs_plan_run_batch (all roots, pinned host "
+                        "level/parent: D2H per root) while the next step's plan (H2D) is built on a second "
+                        "stream"}
 
     # ---- CPU baseline: the oracle, 1 core, bounded sample, rank 0 at N=1 ----
     cpu = None
@@ -645,6 +691,9 @@ def main():
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,
+            "traversed_edges_total": int(te_all),
+            "runs_total": runs_all,
+            "process_group": {"backend": backend, "world_size": world},
             "clocks": clk.summary(),
             "parity": parity,
             "graph_gen_s": round(t_gen, 2),

@@ -236,6 +236,22 @@ void l2_persist_release(int dev)
     }
 }
 
+// Host -> device copy in 32 MiB pieces, for the same reason as d2h_chunked:
+// a plan built from a host CSR while another plan's BFS runs (bench.py's e2e
+// leg builds step k+1's plan during step k) must not hold back that BFS's
+// kernel launches behind one multi-GB copy.
+static cudaError_t h2d_chunked(void *dst, const void *src, size_t bytes, cudaStream_t s)
+{
+    const size_t piece = 32ull << 20;
+    for (size_t off = 0; off < bytes; off += piece) {
+        const size_t nb = bytes - off < piece ? bytes - off : piece;
+        cudaError_t e = cudaMemcpyAsync((char *)dst + off, (const char *)src + off, nb,
+                                        cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
 uint64_t next_pow2(uint64_t x)
 {
     uint64_t c = 1;
@@ -561,12 +577,8 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         p->owns_graph = true;
         e = pool_alloc(&p->row_ptr, (size_t)(n + 1) * sizeof(int64_t), p->stream);
         if (e == cudaSuccess) e = pool_alloc(&p->col, (size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t), p->stream);
-        if (e == cudaSuccess)
-            e = cudaMemcpyAsync(p->row_ptr, gph->row_ptr, (size_t)(n + 1) * sizeof(int64_t),
-                                cudaMemcpyHostToDevice, p->stream);
-        if (e == cudaSuccess && nnz > 0)
-            e = cudaMemcpyAsync(p->col, gph->col, (size_t)nnz * sizeof(int32_t),
-                                cudaMemcpyHostToDevice, p->stream);
+        if (e == cudaSuccess) e = h2d_chunked(p->row_ptr, gph->row_ptr, (size_t)(n + 1) * sizeof(int64_t), p->stream);
+        if (e == cudaSuccess && nnz > 0) e = h2d_chunked(p->col, gph->col, (size_t)nnz * sizeof(int32_t), p->stream);
         if (e != cudaSuccess) return fail(from_cuda(e));
     }
     if (task == kTaskSSSP && nnz > 0) {

@@ -43,13 +43,45 @@ __device__ __forceinline__ bool bench_publish(const tq_device_view &q, unsigned 
     return tq_publish(q, t, item);
 }
 
-// Bounded exponential back-off after a failed CAS (tq_bench_cfg.cas_backoff_ns;
-// 0 = retry at once, the naive form): 32 ns doubling up to bo_max.
+// Bounded, randomised exponential back-off after a failed CAS
+// (tq_bench_cfg.cas_backoff_ns; 0 = retry at once, the naive form), the same
+// two forms as the BFS comparators (bfs.cu): per-thread BASE lanes sit out a
+// random number of ~32 ns retry rounds (lanes of a warp fail together and a
+// sleep would stall the warp as a unit); the AN proxy's warp sleeps a random
+// time in [window/2, window].  The window doubles from 32 ns up to bo_max.
+__device__ __forceinline__ unsigned b_rand()
+{
+    unsigned r;
+    asm volatile("mov.u32 %0, %%globaltimer_lo;" : "=r"(r));
+    r ^= (blockIdx.x * blockDim.x + threadIdx.x) * 0x9E3779B9u;
+    r ^= r >> 15;
+    r *= 0x2C1B3C6Du;
+    r ^= r >> 12;
+    return r;
+}
+struct BLaneBackoff {
+    unsigned win = 0, skip = 0;
+};
+__device__ __forceinline__ bool b_backoff_wait(BLaneBackoff &b)
+{
+    if (!b.skip) return false;
+    --b.skip;
+    __nanosleep(32);
+    return true;
+}
+__device__ __forceinline__ void b_backoff_fail(BLaneBackoff &b, unsigned bo_max)
+{
+    if (!bo_max) return;
+    const unsigned maxw = bo_max / 32 > 1 ? bo_max / 32 : 1;
+    b.win = b.win ? min(2 * b.win, maxw) : 1;
+    b.skip = b_rand() % (b.win + 1);
+}
 __device__ __forceinline__ void b_backoff(unsigned *bo, unsigned bo_max)
 {
     if (!bo_max) return;
     *bo = *bo ? min(*bo * 2, bo_max) : min(32u, bo_max);
-    __nanosleep(*bo);
+    const unsigned r = __shfl_sync(TQ_FULL_MASK, b_rand(), 0);  // one draw per warp
+    __nanosleep(*bo / 2 + r % (*bo / 2 + 1));
 }
 
 // BASE enqueue / dequeue with the ticket returned (for the logs)
@@ -57,8 +89,9 @@ __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t 
                                               unsigned long long *t_out, unsigned *atom, unsigned *fail,
                                               unsigned bo_max)
 {
-    unsigned bo = 0;
+    BLaneBackoff bo;
     for (unsigned tries = 0; tries < (1u << 24); ++tries) {
+        if (b_backoff_wait(bo)) continue;
         const unsigned long long pos = tq_ld_relaxed(q.rear);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -71,7 +104,7 @@ __device__ __forceinline__ bool b_cas_enqueue(const tq_device_view &q, uint32_t 
                 return true;
             }
             ++*fail;
-            b_backoff(&bo, bo_max);
+            b_backoff_fail(bo, bo_max);
         } else if (dif < 0) {
             tq_status_set_thread(q, TQ_ABORTED_FULL);
             return false;
@@ -85,8 +118,9 @@ __device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *
                                              unsigned long long *t_out, unsigned *atom, unsigned *fail,
                                              unsigned bo_max)
 {
-    unsigned bo = 0;
+    BLaneBackoff bo;
     for (unsigned tries = 0; tries < (1u << 12); ++tries) {
+        if (b_backoff_wait(bo)) continue;
         const unsigned long long pos = tq_ld_relaxed(q.front);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -100,7 +134,7 @@ __device__ __forceinline__ int b_cas_dequeue(const tq_device_view &q, uint32_t *
                 return 1;
             }
             ++*fail;
-            b_backoff(&bo, bo_max);
+            b_backoff_fail(bo, bo_max);
         } else if (dif < 0) {
             return 0;
         }

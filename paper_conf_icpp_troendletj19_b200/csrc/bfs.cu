@@ -177,13 +177,50 @@ __device__ __forceinline__ T warp_sum(T x)
 // CAS-based comparison queues (BASE and AN)
 // ---------------------------------------------------------------------------
 
-// Bounded exponential back-off after a failed CAS (bfs_opts.cas_backoff_ns;
-// 0 = retry at once, the naive form): 32 ns doubling up to bo_max.
+__device__ __forceinline__ unsigned backoff_rand()
+{
+    unsigned r;
+    asm volatile("mov.u32 %0, %%globaltimer_lo;" : "=r"(r));
+    r ^= (blockIdx.x * blockDim.x + threadIdx.x) * 0x9E3779B9u;
+    r ^= r >> 15;
+    r *= 0x2C1B3C6Du;
+    r ^= r >> 12;
+    return r;
+}
+
+// Bounded, randomised exponential back-off after a failed CAS
+// (bfs_opts.cas_backoff_ns; 0 = retry at once, the naive form).
+//
+// Per-thread form (BASE): the 32 lanes of a warp fail together in lock-step
+// (one CAS of the 32 wins), and a sleep would stall the warp as a unit, so a
+// lane instead sits out a random number of ~32 ns retry rounds in a window
+// that doubles per failure up to bo_max ns: only lanes whose wait expired
+// issue the next CAS.
+struct LaneBackoff {
+    unsigned win = 0, skip = 0;
+};
+__device__ __forceinline__ bool backoff_wait(LaneBackoff &b)
+{
+    if (!b.skip) return false;
+    --b.skip;
+    __nanosleep(32);
+    return true;
+}
+__device__ __forceinline__ void backoff_fail(LaneBackoff &b, unsigned bo_max)
+{
+    if (!bo_max) return;
+    const unsigned maxw = bo_max / 32 > 1 ? bo_max / 32 : 1;
+    b.win = b.win ? min(2 * b.win, maxw) : 1;
+    b.skip = backoff_rand() % (b.win + 1);
+}
+// Warp form (AN, the proxy's CAS): the warp sleeps a random time in
+// [window/2, window], the window doubling from 32 ns up to bo_max ns.
 __device__ __forceinline__ void cas_backoff(unsigned *bo, unsigned bo_max)
 {
     if (!bo_max) return;
     *bo = *bo ? min(*bo * 2, bo_max) : min(32u, bo_max);
-    __nanosleep(*bo);
+    const unsigned r = __shfl_sync(TQ_FULL_MASK, backoff_rand(), 0);  // one draw per warp
+    __nanosleep(*bo / 2 + r % (*bo / 2 + 1));
 }
 
 // BASE dequeue of one item by one lane: a classic bounded CAS queue (per-slot
@@ -191,8 +228,9 @@ __device__ __forceinline__ void cas_backoff(unsigned *bo, unsigned bo_max)
 __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_t *item,
                                                 unsigned *atom, unsigned *fail, unsigned bo_max)
 {
-    unsigned bo = 0;
+    LaneBackoff bo;
     for (unsigned tries = 0; tries < kMaxDeqRetries; ++tries) {
+        if (backoff_wait(bo)) continue;
         const unsigned long long pos = tq_ld_relaxed(q.front);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -205,7 +243,7 @@ __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_
                 return true;
             }
             ++*fail;
-            cas_backoff(&bo, bo_max);
+            backoff_fail(bo, bo_max);
         } else if (dif < 0) {
             return false;  // queue empty: the exception BASE retries on
         }
@@ -217,8 +255,9 @@ __device__ __forceinline__ bool cas_dequeue_one(const tq_device_view &q, uint32_
 __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_t item,
                                                 unsigned *atom, unsigned *fail, unsigned bo_max)
 {
-    unsigned bo = 0;
+    LaneBackoff bo;
     for (unsigned tries = 0; tries < kMaxEnqRetries; ++tries) {
+        if (backoff_wait(bo)) continue;
         const unsigned long long pos = tq_ld_relaxed(q.rear);
         unsigned long long *s = q.slots + (pos & q.mask);
         const unsigned long long v = tq_ld_relaxed(s);
@@ -230,7 +269,7 @@ __device__ __forceinline__ bool cas_enqueue_one(const tq_device_view &q, uint32_
                 return true;
             }
             ++*fail;
-            cas_backoff(&bo, bo_max);
+            backoff_fail(bo, bo_max);
         } else if (dif < 0) {
             tq_status_set_thread(q, TQ_ABORTED_FULL);
             return false;
@@ -344,13 +383,22 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
     if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
         unsigned long long base;
         if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
-            base = tq_warp_reserve_rear(q, cnt, qatom);
+            // the proxy's AFA is issued, then the release fence, and
+            // only then is the reserved base read: the fence's drain of this
+            // warp's earlier stores overlaps the atomic's round trip
+            unsigned long long b0 = 0;
+            if (lane == 0) {
+                b0 = tq_atom_add(q.rear, (unsigned long long)cnt);
+                ++*qatom;
+            }
+            // release: the W updates (and this warp's Rear reservation) are
+            // ordered before the tokens that name them
+            tq_fence_release();
+            base = tq_shfl64(b0, 0);
         } else {
             if (!an_reserve_rear(q, cnt, &base, qatom, casfail, bo_max)) return;
+            tq_fence_release();  // as above
         }
-        // release: the W updates (and this warp's Rear reservation) are
-        // ordered before the tokens that name them
-        tq_fence_release();
         if (VARIANT == TQ_VARIANT_RF_AN && base + cnt <= lap_end) {  // warp-uniform
             for (unsigned i = lane; i < cnt; i += 32) {
                 const unsigned long long t = base + i;
@@ -409,14 +457,18 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
     } else {
         unsigned long long base;
         if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
-            base = tq_warp_reserve_rear(q, n, qatom);
-        } else if constexpr (VARIANT == TQ_VARIANT_AN) {
-            if (!an_reserve_rear(q, n, &base, qatom, casfail, bo_max)) return;
-        }
-        if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
+            unsigned long long b0 = 0;  // AFA, then the fence, then its result (as in enqueue_staged)
+            if (lane == 0) {
+                b0 = tq_atom_add(q.rear, (unsigned long long)n);
+                ++*qatom;
+            }
             // release: a chunk token names the hub's W entry (its level), and
             // this warp's Rear reservation is ordered before its Done increment
             tq_fence_release();
+            base = tq_shfl64(b0, 0);
+        } else if constexpr (VARIANT == TQ_VARIANT_AN) {
+            if (!an_reserve_rear(q, n, &base, qatom, casfail, bo_max)) return;
+            tq_fence_release();  // as above
         } else {  // PER_THREAD_AFA: each lane reserves its own share
             const unsigned mine = lane < n ? (n - lane + 31) / 32 : 0;
             base = 0;

@@ -43,7 +43,7 @@ def gather(vec, dist=None, device=None):
     """All-gather the per-rank summaries; returns a (world, len(STAT_KEYS)) list."""
     import torch
     t = torch.tensor(vec, dtype=torch.float64, device=device)
-    if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
+    if dist is None or not dist.is_initialized():
         return [t.tolist()]
     world = dist.get_world_size()
     out = torch.empty(world * t.numel(), dtype=torch.float64, device=device)
