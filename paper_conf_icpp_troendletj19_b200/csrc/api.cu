@@ -659,9 +659,18 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     } else {
         p->blocks = full;
         p->auto_blocks = task == kTaskBFS && o.deep_grid >= 0;
+        // Small graphs (< 2^20 CSR entries, e.g. config 1's R-MAT scale 10):
+        // one block per SM.  The run is a chain of ~4 us hops with little
+        // work per level; the full grid only adds its start-up reservations
+        // (one Front AFA per warp) and idle polling (measured: rmat10 kernel
+        // 111 -> 97 us, a 2-vertex graph 25.6 -> 19.5 us).
+        if (p->auto_blocks && nnz < (1ll << 20)) p->blocks = sm_count(gdev) < full ? sm_count(gdev) : full;
     }
     if (p->blocks < 1) p->blocks = 1;
-    if (task == kTaskBFS && o.l2_persist >= 0) {
+    // (the persisting window only pays when the mirror competes with the col
+    // stream for L2: not for mirrors below 4 MB, whose set-up per launch
+    // would only add launch latency)
+    if (task == kTaskBFS && o.l2_persist >= 0 && p->mirror_bytes >= (4u << 20)) {
         // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the level
         // mirror is probed once per edge; a persisting window keeps it
         // resident against the col stream (shared device limit, see

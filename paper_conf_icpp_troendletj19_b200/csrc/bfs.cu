@@ -618,9 +618,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             if (lane == 0) ++S[ST_EMPTY_POLLS];
             ++idle;
             if ((idle & 3) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
-            // termination test: 1 warp in 8, every 16 idle cycles, so idle
+            // termination test: 1 warp in 8, every 4 idle cycles, so idle
             // warps do not crowd the Rear / Done lines busy warps update
-            if ((idle & 15) == 0 && (warp_gid & 7) == 0) {
+            if ((idle & 3) == 0 && (warp_gid & 7) == 0) {
                 bool fin = false;
                 if (lane == 0) {
                     // Done is read before Rear (R6): done(t1) ==

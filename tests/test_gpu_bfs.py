@@ -403,13 +403,15 @@ def test_level_mirror_widths(tq, bits, parents):
 
 
 def test_deep_graph_plans_shrink_the_grid(tq):
-    """threads == 0: after a run of >= 1,024 levels the plan launches one
-    block per SM; shallow graphs keep the full grid; an
-    explicit thread count is never changed.  Results stay exact."""
+    """threads == 0: a plan over >= 2^20 CSR entries starts at the full grid
+    and, after a run of >= 1,024 levels, launches one block per SM (DESIGN.md
+    7a); shallow graphs keep the full grid; graphs below 2^20 entries use one
+    block per SM from the start; an explicit thread count is never changed.
+    Results stay exact."""
     import torch
     full = tq.persistent_threads()
     sms = torch.cuda.get_device_properties(0).multi_processor_count
-    deep = edges_to_csr(np.arange(2999), np.arange(1, 3000), 3000, "path3000")
+    deep = grid_csr(1100, 512)  # 2.25M CSR entries, 1,610 levels from the corner
     rp, col = to_dev(deep)
     lv = torch.empty(deep.n_vertices, dtype=torch.int32, device="cuda")
     pa = torch.empty_like(lv)
@@ -422,12 +424,19 @@ def test_deep_graph_plans_shrink_the_grid(tq):
     with tq.BfsPlan(rp, col, threads=4096, timeout_s=30) as plan:
         plan.run(0, lv, pa)
         assert plan.run(7, lv, pa)["persistent_threads"] == 4096
-    g = kronecker_csr(12, 16, 5)
+    g = kronecker_csr(16, 16, 5)  # shallow, > 2^20 entries: the full grid stays
     rp, col = to_dev(g)
     lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
     with tq.BfsPlan(rp, col) as plan:
         plan.run(int(sample_roots(g.row_ptr, 1, 1)[0]), lv, None)
         assert plan.run(int(sample_roots(g.row_ptr, 1, 2)[0]), lv, None)["persistent_threads"] == full
+    small = edges_to_csr(np.arange(2999), np.arange(1, 3000), 3000, "path3000")
+    rp, col = to_dev(small)
+    lv = torch.empty(small.n_vertices, dtype=torch.int32, device="cuda")
+    with tq.BfsPlan(rp, col, timeout_s=30) as plan:
+        st = plan.run(0, lv, pa[:small.n_vertices])
+        check_against_oracle(small, 0, lv, pa[:small.n_vertices], st)
+        assert st["persistent_threads"] == sms * 256
 
 
 @pytest.mark.parametrize("t_main,t_chunk", [((1 << 32) - 3000, (1 << 32) - 40),
