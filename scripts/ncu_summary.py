@@ -36,6 +36,40 @@ def main(path):
     for v, h in sorted(st, reverse=True)[:10]:
         print(f"{h:40s} {100.0 * v / tot:7.2f}%")
 
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+
+    def num(k):
+        try:
+            return float(d[k][0].replace(",", "")) * scale.get(d[k][1], 1)
+        except (KeyError, ValueError):
+            return 0.0
+    # L2 sector lookups from the SMs by the kernel's L2 eviction policy: the
+    # col stream is the only evict_first load, the level-mirror probes the only
+    # evict_last loads; evict_normal = every per-task access (row_ptr, W, x8,
+    # queue slots, chunk table); plus atomics, reductions and stores.  A miss
+    # is a 32-byte sector fetched from DRAM or from the other die's L2.
+    print("--- L2 sector lookups from the SMs, by access class (per launch) ---")
+    cls = [("col stream (evict_first loads)", "lts__t_sectors_srcunit_tex_op_read_evict_first_lookup_hit.sum",
+            "lts__t_sectors_srcunit_tex_op_read_evict_first_lookup_miss.sum"),
+           ("level-mirror probes (evict_last loads)", "lts__t_sectors_srcunit_tex_op_read_evict_last_lookup_hit.sum",
+            "lts__t_sectors_srcunit_tex_op_read_evict_last_lookup_miss.sum"),
+           ("per-task loads (evict_normal)", "lts__t_sectors_srcunit_tex_op_read_evict_normal_lookup_hit.sum",
+            "lts__t_sectors_srcunit_tex_op_read_evict_normal_lookup_miss.sum"),
+           ("atomics (W atomicMin, queue AFAs, nibble CAS)", "lts__t_sectors_srcunit_tex_op_atom_dot_alu_lookup_hit.sum",
+            "lts__t_sectors_srcunit_tex_op_atom_dot_alu_lookup_miss.sum"),
+           ("stores (slots, mirror, markers)", "lts__t_sectors_srcunit_tex_op_write_lookup_hit.sum",
+            "lts__t_sectors_srcunit_tex_op_write_lookup_miss.sum")]
+    tot_miss = 0.0
+    for name, hk, mk in cls:
+        h, m = num(hk), num(mk)
+        tot_miss += m
+        print(f"{name:48s} lookups {h + m:14.0f}  hits {h:14.0f}  misses {m:14.0f}  "
+              f"miss bytes {m * 32 / 1e9:7.3f} GB")
+    print(f"{'cross-die (ltcfabric) sector lookups':48s} {num('lts__t_sectors_srcunit_ltcfabric.sum'):14.0f}")
+    print(f"{'DRAM read / write':48s} {num('dram__bytes_read.sum') / 1e9:8.3f} GB / "
+          f"{num('dram__bytes_write.sum') / 1e9:8.3f} GB   (sum of SM-side miss sectors x 32 B: "
+          f"{tot_miss * 32 / 1e9:.3f} GB)")
+
 
 if __name__ == "__main__":
     main(sys.argv[1])
