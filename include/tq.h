@@ -193,6 +193,14 @@ typedef struct {
     int deep_grid;      /* threads == 0 only: 0 = default on (after a run of
                            >= 1,024 levels later runs use one block per SM),
                            < 0 = always the full persistent grid            */
+    int ticket_lanes;   /* RF_AN: lanes per warp that hold a main-queue ticket
+                           (each holds one DequeueThreadSlotIndex);
+                           0 = auto: 32; 2 on graphs below 2^20 CSR entries
+                           (consecutive tickets -- a level's consecutive
+                           tokens -- then spread over 16x more warps); 8
+                           after the plan dropped to the deep-graph grid
+                           (see threads); 1..32 = exactly that many; else
+                           TQ_ERR_INVALID                                    */
     int l2_persist;     /* 0 = default on: the level mirror is launched with a
                            persisting-L2 access-policy window (the device's
                            persisting limit is raised while any such plan

@@ -42,7 +42,8 @@ class bfs_opts(ctypes.Structure):
                 ("timeout_s", c_dbl), ("backoff_ns", ctypes.c_int), ("device", ctypes.c_int),
                 ("parent_rule", ctypes.c_int), ("hub_queue", ctypes.c_int),
                 ("debug_delay_ns", ctypes.c_int), ("debug_delay_seed", c_u32),
-                ("cas_backoff_ns", ctypes.c_int), ("mirror_bits", ctypes.c_int), ("deep_grid", ctypes.c_int), ("l2_persist", ctypes.c_int)]
+                ("cas_backoff_ns", ctypes.c_int), ("mirror_bits", ctypes.c_int), ("deep_grid", ctypes.c_int),
+                ("ticket_lanes", ctypes.c_int), ("l2_persist", ctypes.c_int)]
 
 
 class bfs_stats(ctypes.Structure):

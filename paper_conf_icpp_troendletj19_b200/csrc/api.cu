@@ -320,6 +320,8 @@ struct bfs_plan {
     bool dirty = false;
     int32_t *out_scratch = nullptr;           // for host outputs
     int cas_backoff_ns = 0;                   // CAS variants: bounded back-off (bfs_opts)
+    int ticket_lanes = 32;                    // RF/AN: lanes per warp holding main-queue tickets
+    bool auto_lanes = false;                  // ticket_lanes chosen by the plan (bfs_opts.ticket_lanes == 0)
     int delay_ns = 0;                         // test only (bfs_opts.debug_delay_ns)
     uint32_t delay_seed = 0;
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -666,6 +668,15 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         // 111 -> 97 us, a 2-vertex graph 25.6 -> 19.5 us).
         if (p->auto_blocks && nnz < (1ll << 20)) p->blocks = sm_count(gdev) < full ? sm_count(gdev) : full;
     }
+    // lanes per warp holding main-queue tickets (bfs_opts.ticket_lanes)
+    if (o.ticket_lanes < 0 || o.ticket_lanes > 32) return fail(TQ_ERR_INVALID);
+    // auto: 32; 2 on graphs below 2^20 CSR entries (rmat10 91 -> 42 us, kron14
+    // 141 -> 83 us); 8 once a plan has dropped to the deep-graph grid (grid
+    // 4096^2 43.4 -> 41.9 ms); large shallow graphs keep 32 (kron24 with 16 /
+    // 8 / 4 lanes: +8% / +19% / +38%) -- results/small_graph_latency_lanes_r02.jsonl,
+    // results/ab_round2_r02.md
+    p->auto_lanes = o.ticket_lanes == 0;
+    p->ticket_lanes = o.ticket_lanes ? o.ticket_lanes : (nnz < (1ll << 20) ? 2 : 32);
     if (p->blocks < 1) p->blocks = 1;
     // (the persisting window only pays when the mirror competes with the col
     // stream for L2: not for mirrors below 4 MB, whose set-up per launch
@@ -739,6 +750,7 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.l2_window_bytes = p->l2_window;
     bp.delay_ns = (unsigned)p->delay_ns;
     bp.cas_backoff_ns = (unsigned)p->cas_backoff_ns;
+    bp.ticket_lanes = p->ticket_lanes >= 32 ? 0xFFFFFFFFu : ((1u << p->ticket_lanes) - 1u);
     bp.delay_seed = p->delay_seed;
     // every slot of [t0, t0 + C) holds "empty for t" when a run starts (after
     // a reset, or at Rear after a finished run; see plan_finish)
@@ -817,6 +829,7 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
     if (p->auto_blocks && status == TQ_FINISHED && p->stats_h[ST_MAX_LEVEL] >= 1024) {
         const int deep_blocks = sm_count(p->device);
         if (p->blocks > deep_blocks) p->blocks = deep_blocks;
+        if (p->auto_lanes && p->ticket_lanes > 8) p->ticket_lanes = 8;
     }
     if (status == TQ_FINISHED) return TQ_OK;
     if (status == TQ_ABORTED_FULL) return TQ_ERR_QUEUE_FULL;

@@ -548,10 +548,13 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     unsigned tk1 = 0, pend1_base = 0, pend1_mask = 0;
     bool have1 = false;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
-        pend_mask = TQ_FULL_MASK;
+        // lanes that hold main-queue tickets (all 32, or the first few on small
+        // graphs, so that a level's consecutive tokens spread over more warps;
+        // a lane outside the mask never becomes hungry)
+        pend_mask = p.ticket_lanes;
         pend1_mask = q1_lanes;
         if (lane == 0) {
-            pend_base = (unsigned)tq_atom_add(q.front, 32ull);
+            pend_base = (unsigned)tq_atom_add(q.front, (unsigned long long)__popc(p.ticket_lanes));
             ++st_qatom;
             if (hubq) {
                 pend1_base = (unsigned)tq_atom_add(q1.front, (unsigned long long)__popc(q1_lanes));

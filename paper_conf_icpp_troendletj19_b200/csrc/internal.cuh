@@ -97,6 +97,7 @@ struct BfsParams {
     unsigned long long q_lap_end;
     unsigned long long q1_lap_end;
     unsigned cas_backoff_ns;   // CAS variants: max back-off after a failed CAS (0 = none)
+    unsigned ticket_lanes;     // RF/AN: mask of the lanes that hold main-queue tickets
 };
 
 // bfs.cu

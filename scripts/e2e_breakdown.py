@@ -54,13 +54,15 @@ for rep in range(2):
     out[f"create_host_csr_s_{rep}"] = round(t1 - t0, 3)
     plan.run(roots[0], lv_d, pa_d)
     t0 = tick()
-    plan.run_batch(roots, lv_d, pa_d, stride=0)
+    sts = plan.run_batch(roots, lv_d, pa_d, stride=0)
     t1 = tick()
     out[f"batch_dev_out_ms_per_root_{rep}"] = round((t1 - t0) / len(roots) * 1e3, 2)
+    out[f"batch_dev_out_event_ms_per_root_{rep}"] = round(sum(s["ms"] for s in sts) / len(roots), 2)
     t0 = tick()
-    plan.run_batch(roots, lv_pin.numpy(), pa_pin.numpy(), stride=0)
+    sts = plan.run_batch(roots, lv_pin.numpy(), pa_pin.numpy(), stride=0)
     t1 = tick()
     out[f"batch_host_out_ms_per_root_{rep}"] = round((t1 - t0) / len(roots) * 1e3, 2)
+    out[f"batch_host_out_event_ms_per_root_{rep}"] = round(sum(s["ms"] for s in sts) / len(roots), 2)
     t0 = time.perf_counter()
     plan.close()
     out[f"destroy_s_{rep}"] = round(time.perf_counter() - t0, 3)

@@ -1,6 +1,8 @@
 """Fixed and per-level latency of one BFS on tiny graphs (config 1 regime):
 kernel and device time (median of 30) for a 2-vertex edge, paths of 10 / 100,
-a 1,000-leaf star and R-MAT scale 10, at several persistent thread counts."""
+a 1,000-leaf star, R-MAT scale 10 and Kronecker scale 14, at several
+persistent thread counts and ticket-holding lanes per warp (argv[1], e.g.
+"0,1,4,32"; 0 = the plan's automatic choice)."""
 import json
 import os
 import statistics
@@ -21,15 +23,19 @@ graphs = {
 }
 g = kronecker_csr(10, 16, 1)
 graphs["rmat10"] = (g, int(sample_roots(g.row_ptr, 1, 2)[0]))
+g = kronecker_csr(14, 16, 1)
+graphs["kron14"] = (g, int(sample_roots(g.row_ptr, 1, 2)[0]))
+LANES = [int(x) for x in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["0"])]
 for name, (g, root) in graphs.items():
     rp, col = torch.from_numpy(g.row_ptr).cuda(), torch.from_numpy(g.col).cuda()
     lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
-    for th in (1024, 37888, 0):
-        with tq.BfsPlan(rp, col, threads=th) as plan:
+    for th, tl in [(th, tl) for th in (1024, 37888, 0) for tl in LANES]:
+        with tq.BfsPlan(rp, col, threads=th, ticket_lanes=tl) as plan:
             for _ in range(3):
                 plan.run(root, lv, None)
             sts = [plan.run(root, lv, None) for _ in range(30)]
-        print(json.dumps({"graph": name, "threads": sts[0]["persistent_threads"], "levels": sts[0]["max_level"] + 1,
+        print(json.dumps({"graph": name, "threads": sts[0]["persistent_threads"], "ticket_lanes": tl,
+                          "levels": sts[0]["max_level"] + 1,
                           "kernel_us": round(statistics.median(s["ms_kernel"] for s in sts) * 1e3, 1),
                           "dev_us": round(statistics.median(s["ms"] for s in sts) * 1e3, 1),
                           "empty_polls": sts[0]["empty_polls"], "tasks": sts[0]["tasks"]}), flush=True)

@@ -475,3 +475,27 @@ def test_set_tickets_argument_checks(tq):
             plan.set_tickets(1 << 62, 0)
         with pytest.raises(tq.TQError):
             plan.set_tickets(0, 1 << 63)
+
+
+@pytest.mark.parametrize("lanes", [1, 3, 17, 32])
+@pytest.mark.parametrize("parents", ["any", "min_id"])
+def test_ticket_lanes(tq, lanes, parents):
+    """bfs_opts.ticket_lanes: only the first `lanes` lanes of a warp hold
+    main-queue tickets (the default picks fewer on small graphs); results stay
+    exact for any count, also with delay injection."""
+    import torch
+    graphs = [kronecker_csr(12, 16, 2), grid_csr(50, 31), tree4_csr(3000)]
+    for g in graphs:
+        rp, col = to_dev(g)
+        lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+        pa = torch.empty_like(lv)
+        root = int(sample_roots(g.row_ptr, 1, 5)[0])
+        with tq.BfsPlan(rp, col, parents=parents, ticket_lanes=lanes, timeout_s=20) as plan:
+            st = plan.run(root, lv, pa)
+            check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
+        with tq.BfsPlan(rp, col, parents=parents, ticket_lanes=lanes, timeout_s=20, debug_delay_ns=2000,
+                        debug_delay_seed=lanes) as plan:
+            st = plan.run(root, lv, pa)
+            check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
+    with pytest.raises(tq.TQError):
+        tq.bfs(rp, col, 0, ticket_lanes=33)
