@@ -549,9 +549,11 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     bool have1 = false;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
         // lanes that hold main-queue tickets (all 32, or the first few on small
-        // graphs, so that a level's consecutive tokens spread over more warps;
-        // a lane outside the mask never becomes hungry)
-        pend_mask = p.ticket_lanes;
+        // graphs, so that a level's consecutive tokens spread over more warps):
+        // the start-up reservation covers popc(ticket_lanes) tickets and the
+        // consume below ranks only the lanes in the mask (a lane outside it
+        // never becomes hungry)
+        pend_mask = TQ_FULL_MASK;
         pend1_mask = q1_lanes;
         if (lane == 0) {
             pend_base = (unsigned)tq_atom_add(q.front, (unsigned long long)__popc(p.ticket_lanes));
@@ -570,6 +572,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
             if constexpr (VARIANT == TQ_VARIANT_RF_AN) {
                 if (pend_mask) {  // Listing 1 lines 16-19
+                    pend_mask &= p.ticket_lanes;
                     const unsigned base = __shfl_sync(TQ_FULL_MASK, pend_base, 0);
                     if (pend_mask >> lane & 1u) {
                         tk = base + __popc(pend_mask & tq_lanemask_lt());
