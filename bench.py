@@ -541,10 +541,16 @@ def main():
     alg_bytes = algorithmic_bytes(te_all, reached_all) / runs_all
     avg_kernel_s = kern_ms_all / runs_all * 1e-3
     achieved = alg_bytes / avg_kernel_s / 1e9
-    traffic = None
+    traffic, traffic_src = None, None
     tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
-    if os.path.exists(tp):
-        traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+    if os.path.exists(tp):  # one committed `ncu --set full` capture of this kernel (per launch)
+        tj = json.load(open(tp))
+        traffic = tj.get("dram_bytes_per_launch")
+        traffic_src = f"profiles/ncu_traffic_{args.workload}.json ({tj.get('capture_round', '?')})"
+    s_last = all_stats[-1] if all_stats else {}
+    kernel_name = ("bfs_persistent_kernel<%s, %s mirror, %d ticket lanes, %d threads>" %
+                   (args.variant.upper(), {8: "byte", 4: "nibble"}.get(s_last.get("mirror_bits"), "?"),
+                    s_last.get("ticket_lanes", 0), s_last.get("persistent_threads", 0)))
 
     probe_roof = None
     if probe_g:
@@ -705,7 +711,7 @@ def main():
                                                  default=tq.persistent_threads(args.variant, device=local))},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak,
                          "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": traffic,
-                         "kernel": "bfs_persistent_kernel<RF_AN>", "peak_source": peak_src,
+                         "traffic_source": traffic_src, "kernel": kernel_name, "peak_source": peak_src,
                          "alg_bytes_per_launch": int(alg_bytes),
                          "avg_launch_ms": round(avg_kernel_s * 1e3, 4)},
             "roofline_l2_probe": probe_roof,

@@ -230,6 +230,8 @@ typedef struct {
                                    marker (already expanded at <= level)      */
     int32_t max_level;
     int32_t persistent_threads;
+    int32_t mirror_bits;        /* level-mirror width of the plan (8 or 4; 0 SSSP) */
+    int32_t ticket_lanes;       /* lanes per warp holding main-queue tickets      */
 } bfs_stats;
 
 /* Single-source BFS.  level_out[v] = hop distance from root (-1 unreached);

@@ -52,7 +52,8 @@ class bfs_stats(ctypes.Structure):
                 ("min_atomics", c_u64), ("reenqueues", c_u64), ("queue_atomics", c_u64),
                 ("cas_failures", c_u64), ("empty_polls", c_u64), ("tickets", c_u64),
                 ("busy_cycles", c_u64), ("rounds", c_u64), ("skipped_tasks", c_u64),
-                ("max_level", c_i32), ("persistent_threads", c_i32)]
+                ("max_level", c_i32), ("persistent_threads", c_i32), ("mirror_bits", c_i32),
+                ("ticket_lanes", c_i32)]
 
 
 class tq_bench_cfg(ctypes.Structure):

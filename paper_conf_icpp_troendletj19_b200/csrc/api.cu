@@ -820,6 +820,8 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
         stats->busy_cycles = h[ST_BUSY_CYCLES];
         stats->rounds = h[ST_ROUNDS];
         stats->persistent_threads = p->blocks * p->block;
+        stats->mirror_bits = p->task == kTaskBFS ? p->mirror_bits : 0;
+        stats->ticket_lanes = p->ticket_lanes;
     }
     // Deep graphs: a BFS of >= 1,024 levels runs a few thousand
     // vertices per level at a time; a full persistent grid then spends L2 on
