@@ -43,17 +43,21 @@ def main(path):
             return float(d[k][0].replace(",", "")) * scale.get(d[k][1], 1)
         except (KeyError, ValueError):
             return 0.0
-    # L2 sector lookups from the SMs by the kernel's L2 eviction policy: the
-    # col stream is the only evict_first load, the level-mirror probes the only
-    # evict_last loads; evict_normal = every per-task access (row_ptr, W, x8,
-    # queue slots, chunk table); plus atomics, reductions and stores.  A miss
-    # is a 32-byte sector fetched from DRAM or from the other die's L2.
-    print("--- L2 sector lookups from the SMs, by access class (per launch) ---")
-    cls = [("col stream (evict_first loads)", "lts__t_sectors_srcunit_tex_op_read_evict_first_lookup_hit.sum",
+    # L2 sector lookups from the SMs by the eviction-policy tag ncu attributes
+    # them to.  The col stream is the only evict_first load and the level-mirror
+    # probes the only evict_last loads, but their createpolicy hints set the
+    # *hit* priority only (the source view lists them as HIT_FIRST/MISS_NORMAL,
+    # HIT_LAST/MISS_NORMAL), so part of their misses are counted under
+    # evict_normal with the per-task loads (row_ptr, W, x8, slots); the per-line
+    # source view (`--page source`, L2 theoretical sectors) is the per-buffer
+    # attribution.  A miss is a 32-byte sector fetched from DRAM or from the
+    # other die's L2.
+    print("--- L2 sector lookups from the SMs, by policy tag (per launch; see comment) ---")
+    cls = [("evict_first-tagged loads (col)", "lts__t_sectors_srcunit_tex_op_read_evict_first_lookup_hit.sum",
             "lts__t_sectors_srcunit_tex_op_read_evict_first_lookup_miss.sum"),
-           ("level-mirror probes (evict_last loads)", "lts__t_sectors_srcunit_tex_op_read_evict_last_lookup_hit.sum",
+           ("evict_last-tagged loads (mirror probes)", "lts__t_sectors_srcunit_tex_op_read_evict_last_lookup_hit.sum",
             "lts__t_sectors_srcunit_tex_op_read_evict_last_lookup_miss.sum"),
-           ("per-task loads (evict_normal)", "lts__t_sectors_srcunit_tex_op_read_evict_normal_lookup_hit.sum",
+           ("evict_normal-tagged loads (per-task; misses)", "lts__t_sectors_srcunit_tex_op_read_evict_normal_lookup_hit.sum",
             "lts__t_sectors_srcunit_tex_op_read_evict_normal_lookup_miss.sum"),
            ("atomics (W atomicMin, queue AFAs, nibble CAS)", "lts__t_sectors_srcunit_tex_op_atom_dot_alu_lookup_hit.sum",
             "lts__t_sectors_srcunit_tex_op_atom_dot_alu_lookup_miss.sum"),
