@@ -508,6 +508,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     // nibble mirror: their probed mirror words (the CAS's expected value)
     __shared__ unsigned cw_all[MIR == 4 ? kWarps : 1][MIR == 4 ? 32 * KU : 1];
     unsigned *cw = cw_all[MIR == 4 ? (threadIdx.x >> 5) : 0];
+    // BFS: the warp's non-empty tokens of the current cycle (edge -> token map)
+    __shared__ uint4 trec_all[TASK == kTaskBFS ? kWarps : 1][32];
+    uint4 *trec = trec_all[TASK == kTaskBFS ? (threadIdx.x >> 5) : 0];
     const tq_device_view q = p.q;
     const unsigned long long cap = q.mask + 1;
     const int chunk = p.chunk;
@@ -787,17 +790,49 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         unsigned cnt = 0;
         const unsigned long long pol_stream = l2_policy_evict_first();
         const unsigned long long pol_keep = l2_policy_evict_last();
-        // Edge -> token map: lane l takes concatenated edges b + 32j + l; its
-        // token is found by a 5-step shuffle binary search over the lanes'
-        // inclusive prefix sums (a shared-memory prefix-max map was measured
-        // and was not faster).
+        // Edge -> token map: lane l takes concatenated edges b + 32j + l.
+        // SSSP finds its token by a 5-step shuffle binary search over the
+        // lanes' inclusive prefix sums; BFS by the rank map below (round 2:
+        // kron24 -1.9%, results/ab_round2_r02.md section 10).
         const unsigned offer_hi = (unsigned)(offer >> 32);  // BFS: the offered level L + 1
+        // BFS edge -> token map without the shuffle search: the warp's
+        // non-empty tokens, in lane order, as {ebase, offered level, lane}
+        // records in shared memory; the token of entry g is the one with the
+        // largest start <= g, found from a bitmask of the token starts inside
+        // each 32-entry slice (one redux.or) plus a running count.
+        const int tstart = incl - deg;
+        if constexpr (TASK == kTaskBFS) {
+            const unsigned ne = __ballot_sync(TQ_FULL_MASK, deg > 0);
+            if (deg > 0)
+                trec[__popc(ne & tq_lanemask_lt())] =
+                    make_uint4((unsigned)ebase, (unsigned)((unsigned long long)ebase >> 32), offer_hi, lane);
+            __syncwarp();
+        }
         for (int b = 0; b < total; b += 32 * KU) {
             int32_t u[KU];
             unsigned long long off[KU];  // SSSP: per-edge offer (dist + w, v)
             unsigned lv1[KU];            // BFS: offered level of each edge's token
             unsigned ownp = 0;           // BFS: owner lane of edge j in byte j
             bool val[KU];
+            if constexpr (TASK == kTaskBFS) {
+                // tokens that start before this round
+                int cb = __popc(__ballot_sync(TQ_FULL_MASK, deg > 0 && tstart < b));
+#pragma unroll
+                for (int j = 0; j < KU; ++j) {
+                    const int sj = b + j * 32;
+                    const int g = sj + (int)lane;
+                    val[j] = g < total;
+                    const unsigned rel = (unsigned)(tstart - sj);
+                    const unsigned bs = __reduce_or_sync(TQ_FULL_MASK, (deg > 0 && rel < 32u) ? (1u << rel) : 0u);
+                    const int r = cb + __popc(bs & (TQ_FULL_MASK >> (31u - lane))) - 1;
+                    cb += __popc(bs);
+                    const uint4 t = trec[r < 0 ? 0 : r];
+                    const long long eb = (long long)(((unsigned long long)t.y << 32) | t.x);
+                    u[j] = val[j] ? ld_nc_i32(p.col + eb + g, pol_stream) : 0;
+                    lv1[j] = t.z;
+                    ownp |= t.w << (8 * j);
+                }
+            } else
 #pragma unroll
             for (int j = 0; j < KU; ++j) {
                 const int g = b + j * 32 + (int)lane;
