@@ -236,13 +236,13 @@ void l2_persist_release(int dev)
     }
 }
 
-// Host -> device copy in 32 MiB pieces, for the same reason as d2h_chunked:
+// Host -> device copy in 4 MiB pieces, for the same reason as d2h_chunked:
 // a plan built from a host CSR while another plan's BFS runs (bench.py's e2e
 // leg builds step k+1's plan during step k) must not hold back that BFS's
 // kernel launches behind one multi-GB copy.
 static cudaError_t h2d_chunked(void *dst, const void *src, size_t bytes, cudaStream_t s)
 {
-    const size_t piece = 32ull << 20;
+    const size_t piece = 4ull << 20;
     for (size_t off = 0; off < bytes; off += piece) {
         const size_t nb = bytes - off < piece ? bytes - off : piece;
         cudaError_t e = cudaMemcpyAsync((char *)dst + off, (const char *)src + off, nb,
@@ -275,12 +275,19 @@ constexpr size_t kCtrBytes = kOffStatus + TQ_STATUS_COPIES * TQ_STATUS_STRIDE * 
 
 struct tq_queue {
     int device = 0;
+    cudaStream_t stream = nullptr;      // creation / free stream (legacy default for tq_create)
     uint64_t cap = 0;
     unsigned log2cap = 0;
     unsigned long long *slots = nullptr;
     char *ctr = nullptr;
     tq_device_view view{};
 };
+
+// Device output buffers of bfs_plan_run_batch with host outputs: a root's
+// D2H copy may take longer than the next root's BFS while both run (the host
+// link is shared with the kernel's traffic), so a ring of three lets the
+// copies fall two roots behind before a BFS has to wait for a free buffer.
+constexpr int kOutBufs = 3;
 
 struct bfs_plan {
     int device = 0;
@@ -312,9 +319,9 @@ struct bfs_plan {
     unsigned long long *stats_h = nullptr;    // pinned
     unsigned long long *ctr_h = nullptr;      // pinned: front, rear, done, rear1, status
     bool in_flight = false;                   // launched, not yet waited for
-    int32_t *dbuf[2] = {nullptr, nullptr};    // batch: double-buffered device outputs
+    int32_t *dbuf[kOutBufs] = {};             // batch: device output buffers (ring)
     cudaStream_t copy_stream = nullptr;       // batch: D2H copies
-    cudaEvent_t bfs_done[2] = {nullptr, nullptr}, copy_done[2] = {nullptr, nullptr};
+    cudaEvent_t bfs_done[kOutBufs] = {}, copy_done[kOutBufs] = {};
     size_t l2_window = 0;                     // persisting-L2 window over the level mirror
     unsigned long long next_ticket = 0;
     bool dirty = false;
@@ -372,7 +379,12 @@ const char *tq_strerror(tq_status s)
 // ------------------------------------------------------------------------
 // queue objects
 // ------------------------------------------------------------------------
-tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
+// Queue creation / destruction on a given stream: the public entry points use
+// the legacy default stream and synchronise the device; a plan uses its own
+// stream and synchronises only that, so a plan built while another plan's BFS
+// runs (bench.py's e2e leg) neither waits for nor serialises with that BFS.
+static tq_status queue_create_on(uint64_t capacity, int device, cudaStream_t s, bool device_sync,
+                                 tq_queue **out)
 {
     if (!out) return TQ_ERR_INVALID;
     *out = nullptr;
@@ -382,14 +394,15 @@ tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
     tq_queue *q = new (std::nothrow) tq_queue;
     if (!q) return TQ_ERR_NOMEM;
     q->device = device;
+    q->stream = s;
     q->cap = next_pow2(capacity);
     while ((1ull << q->log2cap) < q->cap) ++q->log2cap;
-    cudaError_t e = pool_alloc(&q->slots, q->cap * sizeof(unsigned long long), 0);
-    if (e == cudaSuccess) e = pool_alloc(&q->ctr, kCtrBytes, 0);
+    cudaError_t e = pool_alloc(&q->slots, q->cap * sizeof(unsigned long long), s);
+    if (e == cudaSuccess) e = pool_alloc(&q->ctr, kCtrBytes, s);
     if (e != cudaSuccess) {
-        pool_free(q->slots, 0);
-        pool_free(q->ctr, 0);
-        cudaDeviceSynchronize();
+        pool_free(q->slots, s);
+        pool_free(q->ctr, s);
+        device_sync ? cudaDeviceSynchronize() : cudaStreamSynchronize(s);
         delete q;
         return from_cuda(e);
     }
@@ -400,8 +413,8 @@ tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
     q->view.status = (unsigned *)(q->ctr + kOffStatus);
     q->view.mask = q->cap - 1;
     q->view.log2_capacity = q->log2cap;
-    tq_status st = tq_reset(q, nullptr);
-    if (st == TQ_OK) st = from_cuda(cudaDeviceSynchronize());
+    tq_status st = tq_reset(q, s);
+    if (st == TQ_OK) st = from_cuda(device_sync ? cudaDeviceSynchronize() : cudaStreamSynchronize(s));
     if (st != TQ_OK) {
         tq_destroy(q);
         return st;
@@ -410,13 +423,19 @@ tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
     return TQ_OK;
 }
 
+tq_status tq_create(uint64_t capacity, int device, tq_queue **out)
+{
+    return queue_create_on(capacity, device, nullptr, true, out);
+}
+
 tq_status tq_destroy(tq_queue *q)
 {
     if (!q) return TQ_OK;
     DeviceGuard g(q->device);
-    // callers have finished with the queue (plans synchronise first)
-    pool_free(q->slots, 0);
-    pool_free(q->ctr, 0);
+    // callers have finished with the queue (plans synchronise first); the
+    // frees are ordered on the stream the queue was created on
+    pool_free(q->slots, q->stream);
+    pool_free(q->ctr, q->stream);
     delete q;
     return TQ_OK;
 }
@@ -496,7 +515,7 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     pool_free(p->chunk_tab, fs);
     pool_free(p->stats, fs);
     pool_free(p->out_scratch, fs);
-    for (int b = 0; b < 2; ++b) {
+    for (int b = 0; b < kOutBufs; ++b) {
         pool_free(p->dbuf[b], fs);
         if (p->bfs_done[b]) cudaEventDestroy(p->bfs_done[b]);
         if (p->copy_done[b]) cudaEventDestroy(p->copy_done[b]);
@@ -630,7 +649,7 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     uint64_t cap = o.capacity ? o.capacity : next_pow2((uint64_t)((task == kTaskSSSP ? 8 : 2) * n));
     if (cap > (1ull << 31)) cap = 1ull << 31;
     if (!o.capacity && cap < (1ull << 16)) cap = 1ull << 16;
-    tq_status st = tq_create(cap, gdev, &p->q);
+    tq_status st = queue_create_on(cap, gdev, p->stream, false, &p->q);
     if (st != TQ_OK) return fail(st);
     // chunk queue (RF/AN only): a hub emits its chunks at every expansion
     // (one per distinct level, R7); 4x the chunk count, at least 2^20 slots
@@ -648,7 +667,7 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
             if (cap1 < c / 4) cap1 = c / 4;
             if (cap1 < 2) cap1 = 2;
         }
-        st = tq_create(cap1, gdev, &p->q1);
+        st = queue_create_on(cap1, gdev, p->stream, false, &p->q1);
         if (st != TQ_OK) return fail(st);
     }
 
@@ -894,9 +913,9 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
     if (host_l || host_p) {
         // two device output pairs + a copy stream, allocated on first use
         if (!p->dbuf[0]) {
-            for (int b = 0; b < 2; ++b) CK(pool_alloc(&p->dbuf[b], 2 * vb, p->stream));
+            for (int b = 0; b < kOutBufs; ++b) CK(pool_alloc(&p->dbuf[b], 2 * vb, p->stream));
             CK(cudaStreamCreateWithFlags(&p->copy_stream, cudaStreamNonBlocking));
-            for (int b = 0; b < 2; ++b) {
+            for (int b = 0; b < kOutBufs; ++b) {
                 CK(cudaEventCreateWithFlags(&p->bfs_done[b], cudaEventDisableTiming));
                 CK(cudaEventCreateWithFlags(&p->copy_done[b], cudaEventDisableTiming));
                 CK(cudaEventRecord(p->copy_done[b], p->copy_stream));
@@ -911,7 +930,7 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
     // copy enqueued behind the running kernel overlaps it fully.
     int32_t pend = -1;  // root whose outputs still have to be copied
     auto issue_copy = [&](int32_t k) -> cudaError_t {
-        const int b = k & 1;
+        const int b = k % kOutBufs;
         int32_t *lv = level_out + (level_out ? (size_t)k * out_stride : 0);
         int32_t *pa = parent_out + (parent_out ? (size_t)k * out_stride : 0);
         cudaError_t e = cudaStreamWaitEvent(p->copy_stream, p->bfs_done[b], 0);
@@ -928,10 +947,10 @@ tq_status bfs_plan_run_batch(bfs_plan *p, const int32_t *roots, int32_t n_roots,
             if (st == TQ_OK) st = plan_finish(p, stats ? stats + i : nullptr);
             continue;
         }
-        const int b = i & 1;
+        const int b = i % kOutBufs;
         int32_t *dl = lv ? (host_l ? p->dbuf[b] : lv) : nullptr;
         int32_t *dp = pa ? (host_p ? p->dbuf[b] + p->n : pa) : nullptr;
-        // the buffer pair is free once the copy of root i-2 has drained
+        // the buffer pair is free once the copy of root i - kOutBufs has drained
         CK(cudaStreamWaitEvent(p->stream, p->copy_done[b], 0));
         st = plan_launch(p, roots[i], dl, dp);
         if (st != TQ_OK) break;
