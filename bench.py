@@ -574,7 +574,7 @@ def main():
         rp_np, col_np, lv_np, pa_np = rp_pin.numpy(), col_pin.numpy(), lv_pin.numpy(), pa_pin.numpy()
         plan.close()
         torch.cuda.empty_cache()
-        # Step k+1's plan (its 9 GB H2D of the pinned host CSR, in 4 MiB
+        # Step k+1's plan (its 9 GB H2D of the pinned host CSR, in 1 MiB
         # pieces on its own stream) is built by a helper thread while step k's
         # batch runs: every step's H2D and D2H stay inside the timed region,
         # overlapped with the BFS of the neighbouring step (ctypes releases the

@@ -236,13 +236,15 @@ void l2_persist_release(int dev)
     }
 }
 
-// Host -> device copy in 4 MiB pieces, for the same reason as d2h_chunked:
+// Host -> device copy in 1 MiB pieces, for the same reason as d2h_chunked:
 // a plan built from a host CSR while another plan's BFS runs (bench.py's e2e
 // leg builds step k+1's plan during step k) must not hold back that BFS's
-// kernel launches behind one multi-GB copy.
+// kernel launches behind a long copy.  Measured (kron26 e2e step, 9 GB H2D
+// beside 64 BFS): 64 / 16 / 4 / 2 / 1 / 0.5 MiB pieces -> 1.23 / 1.23 / 1.165 /
+// 1.123 / 1.103 / 1.100 s per step (device-only 1.06 s).
 static cudaError_t h2d_chunked(void *dst, const void *src, size_t bytes, cudaStream_t s)
 {
-    const size_t piece = 4ull << 20;
+    const size_t piece = 1ull << 20;
     for (size_t off = 0; off < bytes; off += piece) {
         const size_t nb = bytes - off < piece ? bytes - off : piece;
         cudaError_t e = cudaMemcpyAsync((char *)dst + off, (const char *)src + off, nb,

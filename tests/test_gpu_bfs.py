@@ -499,3 +499,34 @@ def test_ticket_lanes(tq, lanes, parents):
             check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
     with pytest.raises(tq.TQError):
         tq.bfs(rp, col, 0, ticket_lanes=33)
+
+
+def test_persisting_l2_limit_is_reference_counted(tq):
+    """The device-wide persisting-L2 limit is raised by the first plan whose
+    mirror gets an access-policy window and restored only when the last such
+    plan is destroyed (destroying one plan must not reset another's lines)."""
+    import torch
+    from cuda.bindings import runtime as cudart
+    import inputs.gpu as gg
+
+    def limit():
+        err, v = cudart.cudaDeviceGetLimit(cudart.cudaLimit.cudaLimitPersistingL2CacheSize)
+        assert err == cudart.cudaError_t.cudaSuccess
+        return v
+
+    torch.cuda.synchronize()
+    rp, col = gg.kronecker_csr_cuda(23, 8, 1)  # 8M vertices: an 8 MB byte mirror gets a window
+    before = limit()
+    a = tq.BfsPlan(rp, col)
+    raised = limit()
+    assert raised >= 8 << 20 or raised > before
+    b = tq.BfsPlan(rp, col)
+    assert limit() == raised
+    a.close()
+    assert limit() == raised  # b still holds it
+    lv = torch.empty(rp.numel() - 1, dtype=torch.int32, device="cuda")
+    from inputs import sample_roots
+    r = int(sample_roots(rp.cpu().numpy(), 1, 3)[0])
+    b.run(r, lv, None)
+    b.close()
+    assert limit() == before
