@@ -205,6 +205,19 @@ typedef struct {
                            persisting-L2 access-policy window (the device's
                            persisting limit is raised while any such plan
                            exists, shared by reference count); < 0 = off    */
+    int smem_path;      /* RF_AN BFS: 0 = auto (default): a graph whose whole
+                           run state -- CSR (32-bit offsets), packed W,
+                           expanded-level markers and a ring of 2^ceil(log2
+                           (2V)) slots (at least 64, at most `capacity` when
+                           set) -- fits in one block's shared memory (<= ~227
+                           KB, e.g. config 1's R-MAT scale 10) runs as ONE
+                           1024-thread block with the queue in shared memory,
+                           graph load and unpack included (DESIGN.md "Small
+                           graphs"); < 0 = off (always the global-memory
+                           persistent grid); > 0 = required (TQ_ERR_UNSUPPORTED
+                           if the graph does not fit or the variant / task is
+                           not RF_AN BFS).  threads / ticket_lanes / chunk /
+                           hub_queue / mirror_bits do not apply to it       */
 } bfs_opts;
 
 enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };
@@ -232,6 +245,7 @@ typedef struct {
     int32_t persistent_threads;
     int32_t mirror_bits;        /* level-mirror width of the plan (8 or 4; 0 SSSP) */
     int32_t ticket_lanes;       /* lanes per warp holding main-queue tickets      */
+    int32_t smem_path;          /* 1: the run used the shared-memory path         */
 } bfs_stats;
 
 /* Single-source BFS.  level_out[v] = hop distance from root (-1 unreached);

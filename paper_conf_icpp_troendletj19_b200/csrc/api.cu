@@ -333,6 +333,8 @@ struct bfs_plan {
     bool auto_lanes = false;                  // ticket_lanes chosen by the plan (bfs_opts.ticket_lanes == 0)
     int delay_ns = 0;                         // test only (bfs_opts.debug_delay_ns)
     uint32_t delay_seed = 0;
+    bool smem = false;                        // runs on the shared-memory path (bfs_small.cu)
+    unsigned smem_cap = 0;                    // its ring slots
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
 };
 
@@ -699,10 +701,28 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     p->auto_lanes = o.ticket_lanes == 0;
     p->ticket_lanes = o.ticket_lanes ? o.ticket_lanes : (nnz < (1ll << 20) ? 2 : 32);
     if (p->blocks < 1) p->blocks = 1;
+    // Shared-memory path (bfs_opts.smem_path): the
+    // whole run in one block when CSR + W + markers + a ring of 2V slots fit
+    {
+        // (its packed 32-bit W holds 16-bit vertex ids)
+        const bool eligible = task == kTaskBFS && p->variant == TQ_VARIANT_RF_AN && n <= 65535;
+        uint64_t scap = o.capacity ? next_pow2(o.capacity) : next_pow2((uint64_t)(2 * n));
+        if (scap < 64 && !o.capacity) scap = 64;
+        if (scap < 2) scap = 2;
+        const bool fits = eligible && small_smem_bytes(n, nnz, scap) <= small_smem_limit(gdev);
+        if (o.smem_path > 0 && !fits) return fail(TQ_ERR_UNSUPPORTED);
+        if (o.smem_path >= 0 && fits) {
+            p->smem = true;
+            p->smem_cap = (unsigned)scap;
+            // auto lanes: 8 per warp (config 1, 1/2/4/8/32 lanes: 54/.../39/47 us,
+            // results/smem_path_r02.log)
+            if (p->auto_lanes) p->ticket_lanes = 8;
+        }
+    }
     // (the persisting window only pays when the mirror competes with the col
     // stream for L2: not for mirrors below 4 MB, whose set-up per launch
     // would only add launch latency)
-    if (task == kTaskBFS && o.l2_persist >= 0 && p->mirror_bytes >= (4u << 20)) {
+    if (task == kTaskBFS && !p->smem && o.l2_persist >= 0 && p->mirror_bytes >= (4u << 20)) {
         // L2 persistence (B200: up to ~79 MiB of the 126 MB L2): the level
         // mirror is probed once per edge; a persisting window keeps it
         // resident against the col stream (shared device limit, see
@@ -778,13 +798,26 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.q_lap_end = p->next_ticket + (bp.q.mask + 1);
     bp.q1_lap_end = p->hub_queue ? p->next_ticket1 + (bp.q1.mask + 1) : 0ull;
 
-    CK(cudaEventRecord(p->ev[0], s));
-    CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));
-    CK(cudaEventRecord(p->ev[1], s));
-    CK(launch_bfs_persistent(p->variant, bp, p->blocks, p->block, s));
-    CK(cudaEventRecord(p->ev[2], s));
-    CK(launch_bfs_unpack(bp, level, parent, s));
-    CK(cudaEventRecord(p->ev[3], s));
+    bp.nnz = p->nnz;
+    bp.small_cap = p->smem_cap;
+    if (p->smem) {
+        // one launch: graph load, BFS over the shared-memory queue, unpack
+        // (its statistics and status land where the grid path puts them;
+        // the global queues are untouched, so their tickets stay put)
+        CK(cudaEventRecord(p->ev[0], s));
+        CK(cudaEventRecord(p->ev[1], s));
+        CK(launch_bfs_small(bp, root, level, parent, s));
+        CK(cudaEventRecord(p->ev[2], s));
+        CK(cudaEventRecord(p->ev[3], s));
+    } else {
+        CK(cudaEventRecord(p->ev[0], s));
+        CK(launch_bfs_init(bp, root, p->next_ticket, p->next_ticket1, s));
+        CK(cudaEventRecord(p->ev[1], s));
+        CK(launch_bfs_persistent(p->variant, bp, p->blocks, p->block, s));
+        CK(cudaEventRecord(p->ev[2], s));
+        CK(launch_bfs_unpack(bp, level, parent, s));
+        CK(cudaEventRecord(p->ev[3], s));
+    }
     CK(cudaMemcpyAsync(p->stats_h, p->stats, kStatCount * sizeof(unsigned long long),
                        cudaMemcpyDeviceToHost, s));
     unsigned long long *ctr = p->ctr_h;  // pinned: front, rear, done, rear1, status
@@ -836,13 +869,15 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
         stats->reached = h[ST_REACHED];
         stats->traversed_edges = h[ST_DEG_SUM] / 2;
         stats->max_level = (int32_t)h[ST_MAX_LEVEL];
-        stats->tickets = (ctr[1] - t0) + (p->hub_queue ? ctr[3] - t1 : 0ull);
+        stats->tickets = p->smem ? h[ST_SMEM_TICKETS] : (ctr[1] - t0) + (p->hub_queue ? ctr[3] - t1 : 0ull);
         stats->skipped_tasks = h[ST_SKIPPED];
         stats->busy_cycles = h[ST_BUSY_CYCLES];
         stats->rounds = h[ST_ROUNDS];
         stats->persistent_threads = p->blocks * p->block;
         stats->mirror_bits = p->task == kTaskBFS ? p->mirror_bits : 0;
         stats->ticket_lanes = p->ticket_lanes;
+        stats->smem_path = p->smem ? 1 : 0;
+        if (p->smem) stats->persistent_threads = 1024;
     }
     // Deep graphs: a BFS of >= 1,024 levels runs a few thousand
     // vertices per level at a time; a full persistent grid then spends L2 on

@@ -63,6 +63,7 @@ enum StatIndex {
     ST_REACHED,
     ST_DEG_SUM,
     ST_MAX_LEVEL,
+    ST_SMEM_TICKETS,  // shared-memory path: tickets issued (its Rear at the end)
     ST_COUNT_
 };
 
@@ -98,6 +99,8 @@ struct BfsParams {
     unsigned long long q1_lap_end;
     unsigned cas_backoff_ns;   // CAS variants: max back-off after a failed CAS (0 = none)
     unsigned ticket_lanes;     // RF/AN: mask of the lanes that hold main-queue tickets
+    int64_t nnz;               // CSR entries (the shared-memory path loads them all)
+    unsigned small_cap;        // shared-memory path: ring slots (power of two)
 };
 
 // bfs.cu
@@ -110,6 +113,12 @@ cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm);
 cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int32_t *hub_base,
                               int2 **chunk_tab_out, int64_t *n_chunks_out, cudaStream_t s);
 cudaError_t launch_queue_reset(const tq_device_view &q, unsigned long long t0, cudaStream_t s);
+
+// bfs_small.cu: the whole run (load, BFS over a shared-memory queue, unpack)
+// in one 1024-thread block, for graphs whose state fits in shared memory
+size_t small_smem_bytes(int64_t n, int64_t nnz, uint64_t cap);
+size_t small_smem_limit(int dev);
+cudaError_t launch_bfs_small(const BfsParams &p, int32_t root, int32_t *level, int32_t *parent, cudaStream_t s);
 
 // bench.cu
 struct BenchParams {

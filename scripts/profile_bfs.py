@@ -26,4 +26,4 @@ for i in range(args.runs):
     st = plan.run(roots[0], lv, pa, grow_on_full=True)
     print({k: st[k] for k in ("ms", "ms_kernel", "traversed_edges", "reached", "tasks", "chunk_tasks",
                               "edges_scanned", "min_atomics", "reenqueues", "queue_atomics",
-                              "empty_polls", "max_level")})
+                              "empty_polls", "max_level", "busy_cycles", "rounds", "skipped_tasks")})

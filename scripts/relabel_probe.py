@@ -15,7 +15,7 @@ import paper_conf_icpp_troendletj19_b200 as tq
 ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="kron24x8")
 ap.add_argument("--roots", type=int, default=4)
-ap.add_argument("--mode", default="sorted", choices=["sorted", "strided", "compact"])
+ap.add_argument("--mode", default="sorted", choices=["sorted", "strided", "compact", "isorted"])
 ap.add_argument("--hub-shift", type=int, default=7)
 ap.add_argument("--hubs", type=int, default=1 << 17)
 ap.add_argument("--cache", type=int, default=1, help="strided: enable the hub level cache")
@@ -26,8 +26,15 @@ rp, col = bench.make_graph(kind, a, ef, dev)
 roots = bench.pick_roots(kind, rp.cpu().numpy(), nr)[: args.roots]
 n = rp.numel() - 1
 deg = rp[1:] - rp[:-1]
-if args.mode == "sorted":
+if args.mode in ("sorted", "isorted"):
     new2old = torch.sort(deg, descending=True, stable=True).indices
+    if args.mode == "isorted":  # top H ranks interleaved over the region's 128-byte lines
+        H = min(args.hubs, n) // 128 * 128
+        NL = H // 128
+        r = torch.arange(H, device=dev)
+        pos = (r % NL) * 128 + r // NL
+        top = new2old[:H].clone()
+        new2old[pos] = top
     old2new = torch.empty_like(new2old)
     old2new[new2old] = torch.arange(n, device=dev)
 elif args.mode == "compact":  # top-H degree vertices moved to ids 0..H-1 (swaps), the rest unchanged

@@ -14,6 +14,13 @@ from inputs import (edges_to_csr, grid_csr, kronecker_csr, sample_roots, tree4_c
 pytestmark = pytest.mark.gpu
 
 VARIANTS = ["rf_an", "per_thread_afa", "cas_retry", "an"]
+# RF/AN runs of graphs that fit one block's shared memory take the
+# shared-memory path by default (bfs_opts.smem_path);
+# tests on such graphs run both paths: "grid" forces the persistent grid
+# (smem_path = -1), "smem" requires the shared-memory path (smem_path = 1)
+PATHS = {"grid": -1, "smem": 1}
+VARIANT_PATHS = [("rf_an", "grid"), ("rf_an", "smem"), ("per_thread_afa", "grid"), ("cas_retry", "grid"),
+                 ("an", "grid")]
 
 
 @pytest.fixture(scope="module")
@@ -53,47 +60,71 @@ def check_against_oracle(g, root, level, parent, stats=None, min_id=False):
 
 
 @pytest.mark.parametrize("parents", ["any", "min_id"])
-@pytest.mark.parametrize("variant", VARIANTS)
-def test_rmat10_config1_sample_roots(tq, variant, parents):
+@pytest.mark.parametrize("variant,path", VARIANT_PATHS)
+def test_rmat10_config1_sample_roots(tq, variant, path, parents):
     g = kronecker_csr(10, 16, 1)
     rp, col = to_dev(g)
     import torch
     level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
     parent = torch.empty_like(level)
-    with tq.BfsPlan(rp, col, variant=variant, timeout_s=20, parents=parents) as plan:
+    with tq.BfsPlan(rp, col, variant=variant, timeout_s=20, parents=parents, smem_path=PATHS[path]) as plan:
         for root in sample_roots(g.row_ptr, 16, 2):
             st = plan.run(int(root), level, parent)
             check_against_oracle(g, int(root), level, parent, st, min_id=parents == "min_id")
+            assert st["smem_path"] == (path == "smem")
 
 
+@pytest.mark.parametrize("path", ["grid", "smem"])
 @pytest.mark.parametrize("parents", ["any", "min_id"])
-def test_rmat10_all_roots_rf_an(tq, parents):
+def test_rmat10_all_roots_rf_an(tq, parents, path):
     """Every vertex of the config-1 graph as the root, isolated ones included."""
     import torch
     g = kronecker_csr(10, 16, 1)
     rp, col = to_dev(g)
     level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
     parent = torch.empty_like(level)
-    with tq.BfsPlan(rp, col, timeout_s=20, parents=parents) as plan:
+    with tq.BfsPlan(rp, col, timeout_s=20, parents=parents, smem_path=PATHS[path]) as plan:
         for root in range(g.n_vertices):
-            plan.run(root, level, parent)
-            check_against_oracle(g, root, level, parent, min_id=parents == "min_id")
+            st = plan.run(root, level, parent)
+            check_against_oracle(g, root, level, parent, st, min_id=parents == "min_id")
 
 
-@pytest.mark.parametrize("variant", VARIANTS)
-def test_small_closed_form_graphs_min_id(tq, variant):
+def test_smem_path_is_the_default_for_graphs_that_fit(tq):
+    """Auto (smem_path = 0): config 1's graph runs on the shared-memory path
+    (one 1024-thread block), a graph too large for it on the persistent grid;
+    requiring it for a graph that does not fit, or for another variant, is
+    TQ_ERR_UNSUPPORTED."""
+    g = kronecker_csr(10, 16, 1)
+    rp, col = to_dev(g)
+    root = int(sample_roots(g.row_ptr, 1, 2)[0])
+    level, parent, st = tq.bfs(rp, col, root)
+    check_against_oracle(g, root, level, parent, st)
+    assert st["smem_path"] == 1 and st["persistent_threads"] == 1024
+    big = kronecker_csr(13, 16, 1)
+    rpb, colb = to_dev(big)
+    _, _, st = tq.bfs(rpb, colb, int(sample_roots(big.row_ptr, 1, 2)[0]))
+    assert st["smem_path"] == 0
+    for kw in ({}, {"variant": "an"}):
+        with pytest.raises(tq.TQError) as ei:
+            tq.bfs(rpb if not kw else rp, colb if not kw else col, 0, smem_path=1, **kw)
+        assert ei.value.status == -6
+
+
+@pytest.mark.parametrize("variant,path", VARIANT_PATHS)
+def test_small_closed_form_graphs_min_id(tq, variant, path):
     """Closed-form graphs with the min-id rule: parents are unique, so the
     grid / tree / path parents must equal the oracle's (and the formulas)."""
     for g in [edges_to_csr(np.arange(99), np.arange(1, 100), 100, "path100"), grid_csr(48, 31),
               tree4_csr(3000)]:
         rp, col = to_dev(g)
         for root in {0, g.n_vertices // 2}:
-            level, parent, st = tq.bfs(rp, col, root, variant=variant, timeout_s=20, parents="min_id")
+            level, parent, st = tq.bfs(rp, col, root, variant=variant, timeout_s=20, parents="min_id",
+                                       smem_path=PATHS[path])
             check_against_oracle(g, root, level, parent, st, min_id=True)
 
 
-@pytest.mark.parametrize("variant", VARIANTS)
-def test_small_closed_form_graphs(tq, variant):
+@pytest.mark.parametrize("variant,path", VARIANT_PATHS)
+def test_small_closed_form_graphs(tq, variant, path):
     graphs = [
         edges_to_csr(np.arange(99), np.arange(1, 100), 100, "path100"),
         edges_to_csr(np.zeros(999, dtype=np.int64), np.arange(1, 1000), 1000, "star1000"),
@@ -105,7 +136,7 @@ def test_small_closed_form_graphs(tq, variant):
     for g in graphs:
         rp, col = to_dev(g)
         for root in {0, g.n_vertices // 2, g.n_vertices - 1}:
-            level, parent, st = tq.bfs(rp, col, root, variant=variant, timeout_s=20)
+            level, parent, st = tq.bfs(rp, col, root, variant=variant, timeout_s=20, smem_path=PATHS[path])
             check_against_oracle(g, root, level, parent, st)
 
 
@@ -122,7 +153,8 @@ def test_single_vertex_and_isolated_root(tq):
     assert st["reached"] == 1
 
 
-def test_label_correcting_motif(tq):
+@pytest.mark.parametrize("path", ["grid", "smem"])
+def test_label_correcting_motif(tq, path):
     """r-a, r-b, a-c, c-x, b-x: x has level 2 via b, not 3 via a-c (R4).
     Repeated many times so that different schedules occur."""
     # plus a long path hanging off a to slow one side down
@@ -132,13 +164,13 @@ def test_label_correcting_motif(tq):
     g = edges_to_csr(np.array(src), np.array(dst), n)
     rp, col = to_dev(g)
     for _ in range(20):
-        level, parent, st = tq.bfs(rp, col, 0)
+        level, parent, st = tq.bfs(rp, col, 0, smem_path=PATHS[path])
         check_against_oracle(g, 0, level, parent, st)
 
 
 @pytest.mark.parametrize("parents", ["any", "min_id"])
-@pytest.mark.parametrize("variant", ["rf_an", "an"])
-def test_schedule_independence_under_delay_injection(tq, variant, parents):
+@pytest.mark.parametrize("variant,path", [("rf_an", "grid"), ("rf_an", "auto"), ("an", "grid")])
+def test_schedule_independence_under_delay_injection(tq, variant, path, parents):
     """SURVEY §8(c) "schedule independence": with the test-only delay
     injection (bfs_opts.debug_delay_ns) 1/8 of the vertices are expanded late
     and another 1/8 with a level read long before their offers land, for
@@ -154,7 +186,8 @@ def test_schedule_independence_under_delay_injection(tq, variant, parents):
         root = int(sample_roots(g.row_ptr, 1, 3)[0]) if g.n_vertices > 5000 else 0
         for seed in range(4):
             level, parent, st = tq.bfs(rp, col, root, variant=variant, parents=parents, timeout_s=30,
-                                       chunk=64, debug_delay_ns=20000, debug_delay_seed=seed)
+                                       chunk=64, debug_delay_ns=20000, debug_delay_seed=seed,
+                                       smem_path=PATHS.get(path, 0))
             check_against_oracle(g, root, level, parent, st, min_id=parents == "min_id")
 
 
@@ -203,6 +236,27 @@ def test_queue_full_aborts_and_retry_succeeds(tq):
     assert ei.value.status == -4
     level, parent, st = tq.bfs(rp, col, root, capacity=1 << 14)
     check_against_oracle(g, root, level, parent, st)
+
+
+def test_smem_queue_full_aborts_and_retry_succeeds(tq):
+    """The same queue-full exception on the shared-memory ring (P:268 line 25,
+    P:281): a ring of 64 slots overflows from the top hub of config 1's graph;
+    with a larger ring the same run is exact; a plan answering the abort with
+    grow_on_full moves on to a ring too large for shared memory, i.e. to the
+    persistent grid, and is exact too."""
+    g = kronecker_csr(10, 16, 1)
+    rp, col = to_dev(g)
+    root = int(np.argmax(g.degrees()))
+    with pytest.raises(tq.TQError) as ei:
+        tq.bfs(rp, col, root, capacity=64, smem_path=1)
+    assert ei.value.status == -4
+    level, parent, st = tq.bfs(rp, col, root, capacity=4096, smem_path=1)
+    assert st["smem_path"] == 1
+    check_against_oracle(g, root, level, parent, st)
+    with tq.BfsPlan(rp, col, capacity=64) as plan:
+        st = plan.run(root, level, parent, grow_on_full=True)
+        assert plan.regrows >= 1 and st["smem_path"] == 0
+        check_against_oracle(g, root, level, parent, st)
 
 
 def test_concurrent_plans_on_two_streams(tq):
@@ -337,22 +391,29 @@ def test_any_parent_rule_levels_exact_tree_valid(tq, variant):
         assert st["traversed_edges"] == info["traversed_edges"]
 
 
-def test_ring_wraps_within_runs(tq):
+@pytest.mark.parametrize("path,cap", [("grid", 1024), ("smem", 256)])
+def test_ring_wraps_within_runs(tq, path, cap):
     """A queue smaller than one run's ticket count: every run crosses the
     first-lap boundary t0 + C (R18) and the ring wraps many times
-    across consecutive runs on one plan; results stay exact."""
+    across consecutive runs on one plan (the shared-memory ring restarts at
+    ticket 0 each run and wraps within it: on a 48 x 31 grid, whose frontier
+    stays small, ~1,500 tickets per run through 256 slots); results stay
+    exact."""
     import torch
-    g = kronecker_csr(10, 16, 1)
+    g = kronecker_csr(10, 16, 1) if path == "grid" else grid_csr(48, 31)
     rp, col = to_dev(g)
     level = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
     parent = torch.empty_like(level)
-    with tq.BfsPlan(rp, col, capacity=1024, parents="min_id") as plan:
-        tickets = 0
+    with tq.BfsPlan(rp, col, capacity=cap, parents="min_id", smem_path=PATHS[path]) as plan:
+        tickets, wrapped = 0, 0
         for r in sample_roots(g.row_ptr, 12, 5):
-            st = plan.run(int(r), level, parent, grow_on_full=True)
+            st = plan.run(int(r), level, parent, grow_on_full=path == "grid")
             tickets += st["tickets"]
+            wrapped += st["tickets"] > 4 * cap
             check_against_oracle(g, int(r), level, parent, st, min_id=True)
-    assert tickets > 8 * 1024
+    assert tickets > 8 * cap
+    if path == "smem":  # its ring restarts each run: the wrap is within the runs
+        assert wrapped == 12
 
 
 def test_probe_ceiling_measures(tq):
@@ -389,7 +450,7 @@ def test_level_mirror_widths(tq, bits, parents):
     for g in graphs:
         rp, col = to_dev(g)
         roots = [0, int(sample_roots(g.row_ptr, 1, seed=9)[0])]
-        with tq.BfsPlan(rp, col, parents=parents, timeout_s=20, mirror_bits=bits) as plan:
+        with tq.BfsPlan(rp, col, parents=parents, timeout_s=20, mirror_bits=bits, smem_path=-1) as plan:
             import torch
             lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
             pa = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
@@ -397,7 +458,7 @@ def test_level_mirror_widths(tq, bits, parents):
                 st = plan.run(root, lv, pa)
                 check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
         with tq.BfsPlan(rp, col, parents=parents, timeout_s=20, debug_delay_ns=2000,
-                        debug_delay_seed=3, mirror_bits=bits) as plan:
+                        debug_delay_seed=3, mirror_bits=bits, smem_path=-1) as plan:
             st = plan.run(roots[1], lv, pa)
             check_against_oracle(g, roots[1], lv, pa, st, min_id=parents == "min_id")
 
@@ -433,7 +494,7 @@ def test_deep_graph_plans_shrink_the_grid(tq):
     small = edges_to_csr(np.arange(2999), np.arange(1, 3000), 3000, "path3000")
     rp, col = to_dev(small)
     lv = torch.empty(small.n_vertices, dtype=torch.int32, device="cuda")
-    with tq.BfsPlan(rp, col, timeout_s=30) as plan:
+    with tq.BfsPlan(rp, col, timeout_s=30, smem_path=-1) as plan:
         st = plan.run(0, lv, pa[:small.n_vertices])
         check_against_oracle(small, 0, lv, pa[:small.n_vertices], st)
         assert st["persistent_threads"] == sms * 256
@@ -477,9 +538,10 @@ def test_set_tickets_argument_checks(tq):
             plan.set_tickets(0, 1 << 63)
 
 
+@pytest.mark.parametrize("path", ["grid", "auto"])
 @pytest.mark.parametrize("lanes", [1, 3, 17, 32])
 @pytest.mark.parametrize("parents", ["any", "min_id"])
-def test_ticket_lanes(tq, lanes, parents):
+def test_ticket_lanes(tq, lanes, parents, path):
     """bfs_opts.ticket_lanes: only the first `lanes` lanes of a warp hold
     main-queue tickets (the default picks fewer on small graphs); results stay
     exact for any count, also with delay injection."""
@@ -490,11 +552,12 @@ def test_ticket_lanes(tq, lanes, parents):
         lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
         pa = torch.empty_like(lv)
         root = int(sample_roots(g.row_ptr, 1, 5)[0])
-        with tq.BfsPlan(rp, col, parents=parents, ticket_lanes=lanes, timeout_s=20) as plan:
+        sp = PATHS.get(path, 0)
+        with tq.BfsPlan(rp, col, parents=parents, ticket_lanes=lanes, timeout_s=20, smem_path=sp) as plan:
             st = plan.run(root, lv, pa)
             check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
         with tq.BfsPlan(rp, col, parents=parents, ticket_lanes=lanes, timeout_s=20, debug_delay_ns=2000,
-                        debug_delay_seed=lanes) as plan:
+                        debug_delay_seed=lanes, smem_path=sp) as plan:
             st = plan.run(root, lv, pa)
             check_against_oracle(g, root, lv, pa, st, min_id=parents == "min_id")
     with pytest.raises(tq.TQError):
