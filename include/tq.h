@@ -218,6 +218,18 @@ typedef struct {
                            if the graph does not fit or the variant / task is
                            not RF_AN BFS).  threads / ticket_lanes / chunk /
                            hub_queue / mirror_bits do not apply to it       */
+    int relabel;        /* BFS on the persistent grid: renumber the vertices by
+                           descending degree inside the plan (DESIGN.md
+                           "Vertex relabelling"; the top 2^17 ranks dealt over
+                           their 128-byte lines) so that the hubs' mirror
+                           bytes, W words and markers share sectors.  The plan
+                           then owns a relabelled copy of the CSR (4 B per
+                           entry + 16 B per vertex; a host-CSR plan keeps only
+                           that copy and the original offsets).  Outputs,
+                           roots and parent ids stay in the original
+                           numbering (min-id parents too).  0 = auto (default):
+                           on when some vertex has more than `chunk` edges;
+                           < 0 = off; > 0 = on                              */
 } bfs_opts;
 
 enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };
@@ -246,6 +258,7 @@ typedef struct {
     int32_t mirror_bits;        /* level-mirror width of the plan (8 or 4; 0 SSSP) */
     int32_t ticket_lanes;       /* lanes per warp holding main-queue tickets      */
     int32_t smem_path;          /* 1: the run used the shared-memory path         */
+    int32_t relabelled;         /* 1: the plan runs on a relabelled copy (opts)   */
 } bfs_stats;
 
 /* Single-source BFS.  level_out[v] = hop distance from root (-1 unreached);

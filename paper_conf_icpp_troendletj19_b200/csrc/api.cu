@@ -334,6 +334,11 @@ struct bfs_plan {
     int delay_ns = 0;                         // test only (bfs_opts.debug_delay_ns)
     uint32_t delay_seed = 0;
     bool smem = false;                        // runs on the shared-memory path (bfs_small.cu)
+    // vertex relabelling (relabel.cu): row_ptr / col are then the plan-owned
+    // relabelled CSR and row_ptr0 the original offsets (owned if owns_graph)
+    bool relabelled = false;
+    int32_t *new2old = nullptr, *old2new = nullptr;
+    int64_t *row_ptr0 = nullptr;
     unsigned smem_cap = 0;                    // its ring slots
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
 };
@@ -506,7 +511,13 @@ tq_status bfs_plan_destroy(bfs_plan *p)
     if (p->copy_stream) cudaStreamSynchronize(p->copy_stream);
     // stream-ordered frees after everything that used the memory has finished
     cudaStream_t fs = p->stream;
-    if (p->owns_graph) {
+    if (p->relabelled) {
+        pool_free(p->row_ptr, fs);  // the relabelled CSR (plan-owned)
+        pool_free(p->col, fs);
+        pool_free(p->new2old, fs);
+        pool_free(p->old2new, fs);
+        if (p->owns_graph) pool_free(p->row_ptr0, fs);  // (the original col was freed at create)
+    } else if (p->owns_graph) {
         pool_free(p->row_ptr, fs);
         pool_free(p->col, fs);
     }
@@ -590,6 +601,7 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     p->n = n;
     p->nnz = nnz;
 
+    bool smem_auto_lanes = false;
     auto fail = [&](tq_status s) {
         bfs_plan_destroy(p);
         return s;
@@ -618,6 +630,39 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
                 e = cudaMemcpyAsync(p->wgt, weights, (size_t)nnz * sizeof(int32_t), cudaMemcpyHostToDevice,
                                     p->stream);
             if (e != cudaSuccess) return fail(from_cuda(e));
+        }
+    }
+    // Shared-memory path (bfs_opts.smem_path, DESIGN.md "Small graphs"): the
+    // whole run in one block when CSR + W + markers + a ring of 2V slots fit
+    {
+        // (its packed 32-bit W holds 16-bit vertex ids)
+        const bool eligible = task == kTaskBFS && p->variant == TQ_VARIANT_RF_AN && n <= 65535;
+        uint64_t scap = o.capacity ? next_pow2(o.capacity) : next_pow2((uint64_t)(2 * n));
+        if (scap < 64 && !o.capacity) scap = 64;
+        if (scap < 2) scap = 2;
+        const bool fits = eligible && small_smem_bytes(n, nnz, scap) <= small_smem_limit(gdev);
+        if (o.smem_path > 0 && !fits) return fail(TQ_ERR_UNSUPPORTED);
+        if (o.smem_path >= 0 && fits) {
+            p->smem = true;
+            p->smem_cap = (unsigned)scap;
+            smem_auto_lanes = true;  // (ticket lanes below)
+        }
+    }
+    // Vertex relabelling (bfs_opts.relabel, relabel.cu): BFS on the persistent
+    // grid, auto when a vertex has more than `chunk` edges (a degree-skewed
+    // graph; a uniform graph such as the grid keeps its own numbering)
+    if (task == kTaskBFS && !p->smem && o.relabel >= 0 && n < (1ll << 31) - 1) {
+        RelabelOut ro{};
+        e = build_relabel(p->row_ptr, p->col, n, nnz, o.relabel > 0 ? -1 : chunk, &ro, p->stream);
+        if (e != cudaSuccess) return fail(from_cuda(e));
+        if (ro.new2old) {
+            p->relabelled = true;
+            p->row_ptr0 = p->row_ptr;
+            if (p->owns_graph) pool_free(p->col, p->stream);  // only the relabelled entries are read
+            p->row_ptr = ro.row_ptr;
+            p->col = ro.col;
+            p->new2old = ro.new2old;
+            p->old2new = ro.old2new;
         }
     }
     e = pool_alloc(&p->W, (size_t)n * sizeof(unsigned long long), p->stream);
@@ -700,25 +745,10 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     // results/ab_round2_r02.md
     p->auto_lanes = o.ticket_lanes == 0;
     p->ticket_lanes = o.ticket_lanes ? o.ticket_lanes : (nnz < (1ll << 20) ? 2 : 32);
+    // shared-memory path: 8 lanes per warp (config 1, 1/2/4/8/32 lanes:
+    // 54/.../39/47 us, results/smem_path_r02.log)
+    if (smem_auto_lanes && p->auto_lanes) p->ticket_lanes = 8;
     if (p->blocks < 1) p->blocks = 1;
-    // Shared-memory path (bfs_opts.smem_path, DESIGN.md "Small graphs"): the
-    // whole run in one block when CSR + W + markers + a ring of 2V slots fit
-    {
-        // (its packed 32-bit W holds 16-bit vertex ids)
-        const bool eligible = task == kTaskBFS && p->variant == TQ_VARIANT_RF_AN && n <= 65535;
-        uint64_t scap = o.capacity ? next_pow2(o.capacity) : next_pow2((uint64_t)(2 * n));
-        if (scap < 64 && !o.capacity) scap = 64;
-        if (scap < 2) scap = 2;
-        const bool fits = eligible && small_smem_bytes(n, nnz, scap) <= small_smem_limit(gdev);
-        if (o.smem_path > 0 && !fits) return fail(TQ_ERR_UNSUPPORTED);
-        if (o.smem_path >= 0 && fits) {
-            p->smem = true;
-            p->smem_cap = (unsigned)scap;
-            // auto lanes: 8 per warp (config 1, 1/2/4/8/32 lanes: 54/.../39/47 us,
-            // results/smem_path_r02.log)
-            if (p->auto_lanes) p->ticket_lanes = 8;
-        }
-    }
     // (the persisting window only pays when the mirror competes with the col
     // stream for L2: not for mirrors below 4 MB, whose set-up per launch
     // would only add launch latency)
@@ -800,6 +830,10 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
 
     bp.nnz = p->nnz;
     bp.small_cap = p->smem_cap;
+    bp.new2old = p->new2old;
+    bp.old2new = p->old2new;
+    bp.row_ptr0 = p->row_ptr0;
+    bp.pid_orig = p->relabelled && p->parent_rule == TQ_PARENT_MIN_ID;
     if (p->smem) {
         // one launch: graph load, BFS over the shared-memory queue, unpack
         // (its statistics and status land where the grid path puts them;
@@ -877,6 +911,7 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
         stats->mirror_bits = p->task == kTaskBFS ? p->mirror_bits : 0;
         stats->ticket_lanes = p->ticket_lanes;
         stats->smem_path = p->smem ? 1 : 0;
+        stats->relabelled = p->relabelled ? 1 : 0;
         if (p->smem) stats->persistent_threads = 1024;
     }
     // Deep graphs: a BFS of >= 1,024 levels runs a few thousand

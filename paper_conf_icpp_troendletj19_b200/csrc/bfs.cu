@@ -717,6 +717,10 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                 dly = (unsigned)(mix32((unsigned)v ^ p.delay_seed) & 7u);
                 if (dly == 0) __nanosleep(p.delay_ns);
             }
+            // the parent id W records: on a relabelled plan with min-id
+            // parents, v's original id (the minimum must be the one of the
+            // original numbering); else v itself (the unpack translates)
+            const unsigned pid = (TASK == kTaskBFS && p.pid_orig) ? (unsigned)__ldg(p.new2old + v) : (unsigned)v;
             // current cost of the node (Listing 2 line 21), read fresh
             const unsigned L = (unsigned)(tq_ld_relaxed(p.W + v) >> 32);
             if (dly == 1) __nanosleep(p.delay_ns);
@@ -734,7 +738,7 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     }
                 }
             } else {
-            offer = ((unsigned long long)(L + 1) << 32) | (unsigned)v;
+            offer = ((unsigned long long)(L + 1) << 32) | pid;
             if (!(item & CHUNK_FLAG)) {
                 // expanded-level marker (R7): a vertex already
                 // expanded at a level <= L has offered <= L+1 to every
@@ -1078,26 +1082,30 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
     const int64_t n = p.n_vertices;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    // the root's position (its new id on a relabelled plan) and the parent
+    // id W records for it (the original id when W holds original ids)
+    const int32_t rn = p.old2new ? __ldg(p.old2new + root) : root;
+    const uint32_t rpid = p.pid_orig ? (uint32_t)root : (uint32_t)rn;
     // W: 4 entries (32 bytes) per store pair; plan buffers are pool
     // allocations (256-byte aligned)
     const int64_t n4 = n / 4;
     for (int64_t k = tid; k < n4; k += stride) {
         ulonglong2 a = make_ulonglong2(~0ull, ~0ull), b = a;
         const int64_t i = 4 * k;
-        if (root >= i && root < i + 4) {
-            unsigned long long *e = root < i + 2 ? &a.x : &b.x;
-            e[(root - i) & 1] = (unsigned long long)(uint32_t)root;
+        if (rn >= i && rn < i + 4) {
+            unsigned long long *e = rn < i + 2 ? &a.x : &b.x;
+            e[(rn - i) & 1] = (unsigned long long)rpid;
         }
         reinterpret_cast<ulonglong2 *>(p.W + i)[0] = a;
         reinterpret_cast<ulonglong2 *>(p.W + i)[1] = b;
     }
     for (int64_t i = 4 * n4 + tid; i < n; i += stride)
-        p.W[i] = (i == root) ? (unsigned long long)(uint32_t)root : ~0ull;
+        p.W[i] = (i == rn) ? (unsigned long long)rpid : ~0ull;
     if (p.mir) {  // level mirror: bytes (root's = 0) or nibbles (15 = unreached, root's = 0)
         if (p.mirror_bits == 8)
-            fill_ff((uint8_t *)p.mir, n, root, 0x00u, tid, stride);
+            fill_ff((uint8_t *)p.mir, n, rn, 0x00u, tid, stride);
         else
-            fill_ff((uint8_t *)p.mir, (n + 7) / 8 * 4, root >> 1, ~(0xFu << ((root & 1) << 2)), tid, stride);
+            fill_ff((uint8_t *)p.mir, (n + 7) / 8 * 4, rn >> 1, ~(0xFu << ((rn & 1) << 2)), tid, stride);
     }
     if (p.x8) fill_ff(p.x8, p.mirror_bits == 8 ? n : (n + 1) / 2, -1, 0xFFu, tid, stride);  // markers
     if (p.xd) fill_ff(reinterpret_cast<uint8_t *>(p.xd), 4 * n, -1, 0xFFu, tid, stride);
@@ -1106,7 +1114,7 @@ __global__ void bfs_init_kernel(const BfsParams p, int32_t root, unsigned long l
         if (threadIdx.x < kStatCount) p.stats[threadIdx.x] = 0;
         if (threadIdx.x == 0) {
             p.q.slots[t0 & p.q.mask] =
-                ((unsigned long long)(uint32_t)root << 32) | (unsigned)(t0 + 1);
+                ((unsigned long long)(uint32_t)rn << 32) | (unsigned)(t0 + 1);
             *p.q.front = t0;
             *p.q.rear = t0 + 1;
             // Done counts tasks of both queues: termination is
@@ -1130,19 +1138,39 @@ __global__ void __launch_bounds__(256) bfs_unpack_kernel(const BfsParams p, int3
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     unsigned long long reached = 0, degsum = 0;
     unsigned maxl = 0;
+    // outputs and statistics in the original vertex order: on a relabelled
+    // plan vertex o's word is W[old2new[o]] (a gather), its degree from the
+    // original offsets
+    const int32_t *o2n = p.old2new;
+    const int64_t *rp0 = p.row_ptr0 ? p.row_ptr0 : p.row_ptr;
+    // parents recorded as new ids are translated back
+    const int32_t *n2o = p.pid_orig ? nullptr : p.new2old;
     // 4 vertices per thread with 16-byte accesses when every array is 16-byte
     // aligned (HBM-bound: W 8 B + row_ptr 8 B read, level + parent 8 B written
     // per vertex); the scalar loop takes the tail and unaligned outputs
-    const bool vec = ((reinterpret_cast<uintptr_t>(p.W) | reinterpret_cast<uintptr_t>(p.row_ptr) |
-                       reinterpret_cast<uintptr_t>(level) | reinterpret_cast<uintptr_t>(parent)) & 15) == 0;
+    const bool vec = ((reinterpret_cast<uintptr_t>(p.W) | reinterpret_cast<uintptr_t>(rp0) |
+                       reinterpret_cast<uintptr_t>(o2n) | reinterpret_cast<uintptr_t>(level) |
+                       reinterpret_cast<uintptr_t>(parent)) & 15) == 0;
     int64_t done = 0;
     if (vec) {
         const int64_t n4 = n / 4;
         for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n4; k += stride) {
             const int64_t i = 4 * k;
-            const ulonglong2 w01 = *reinterpret_cast<const ulonglong2 *>(p.W + i);
-            const ulonglong2 w23 = *reinterpret_cast<const ulonglong2 *>(p.W + i + 2);
-            const unsigned long long w[4] = {w01.x, w01.y, w23.x, w23.y};
+            unsigned long long w[4];
+            if (o2n) {
+                const int4 m = __ldg(reinterpret_cast<const int4 *>(o2n + i));
+                w[0] = p.W[m.x];
+                w[1] = p.W[m.y];
+                w[2] = p.W[m.z];
+                w[3] = p.W[m.w];
+            } else {
+                const ulonglong2 w01 = *reinterpret_cast<const ulonglong2 *>(p.W + i);
+                const ulonglong2 w23 = *reinterpret_cast<const ulonglong2 *>(p.W + i + 2);
+                w[0] = w01.x;
+                w[1] = w01.y;
+                w[2] = w23.x;
+                w[3] = w23.y;
+            }
             int4 lv, pa;
             int *lvp = &lv.x, *pap = &pa.x;
             bool any = false;
@@ -1151,7 +1179,7 @@ __global__ void __launch_bounds__(256) bfs_unpack_kernel(const BfsParams p, int3
                 const unsigned l = (unsigned)(w[j] >> 32);
                 const bool r = l != 0xffffffffu;
                 lvp[j] = r ? (int32_t)l : -1;
-                pap[j] = r ? (int32_t)(uint32_t)w[j] : -1;
+                pap[j] = r ? (n2o ? __ldg(n2o + (uint32_t)w[j]) : (int32_t)(uint32_t)w[j]) : -1;
                 if (r) {
                     ++reached;
                     maxl = max(maxl, l);
@@ -1161,9 +1189,9 @@ __global__ void __launch_bounds__(256) bfs_unpack_kernel(const BfsParams p, int3
             if (level) *reinterpret_cast<int4 *>(level + i) = lv;
             if (parent) *reinterpret_cast<int4 *>(parent + i) = pa;
             if (any) {
-                const longlong2 r01 = *reinterpret_cast<const longlong2 *>(p.row_ptr + i);
-                const longlong2 r23 = *reinterpret_cast<const longlong2 *>(p.row_ptr + i + 2);
-                const long long r4 = ld_nc_i64(p.row_ptr + i + 4);
+                const longlong2 r01 = *reinterpret_cast<const longlong2 *>(rp0 + i);
+                const longlong2 r23 = *reinterpret_cast<const longlong2 *>(rp0 + i + 2);
+                const long long r4 = ld_nc_i64(rp0 + i + 4);
                 const long long rp[5] = {r01.x, r01.y, r23.x, r23.y, r4};
 #pragma unroll
                 for (int j = 0; j < 4; ++j)
@@ -1173,14 +1201,14 @@ __global__ void __launch_bounds__(256) bfs_unpack_kernel(const BfsParams p, int3
         done = 4 * n4;
     }
     for (int64_t i = done + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-        const unsigned long long w = p.W[i];
+        const unsigned long long w = p.W[o2n ? o2n[i] : i];
         const unsigned l = (unsigned)(w >> 32);
         const bool r = l != 0xffffffffu;
         if (level) level[i] = r ? (int32_t)l : -1;
-        if (parent) parent[i] = r ? (int32_t)(uint32_t)w : -1;
+        if (parent) parent[i] = r ? (n2o ? __ldg(n2o + (uint32_t)w) : (int32_t)(uint32_t)w) : -1;
         if (r) {
             ++reached;
-            degsum += (unsigned long long)(ld_nc_i64(p.row_ptr + i + 1) - ld_nc_i64(p.row_ptr + i));
+            degsum += (unsigned long long)(ld_nc_i64(rp0 + i + 1) - ld_nc_i64(rp0 + i));
             maxl = max(maxl, l);
         }
     }

@@ -100,6 +100,15 @@ struct BfsParams {
     unsigned cas_backoff_ns;   // CAS variants: max back-off after a failed CAS (0 = none)
     unsigned ticket_lanes;     // RF/AN: mask of the lanes that hold main-queue tickets
     int64_t nnz;               // CSR entries (the shared-memory path loads them all)
+    // vertex relabelling (relabel.cu): row_ptr / col above are then the
+    // relabelled CSR; tokens, W, mirror and markers use new ids, W's parent
+    // field original ids; null = no relabelling
+    const int32_t *new2old;
+    const int32_t *old2new;
+    const int64_t *row_ptr0;   // the original row offsets (unpack statistics)
+    int pid_orig;              // W's parent field holds original ids (relabelled
+                               // min-id plans: the kernel reads new2old); else
+                               // the plan's own ids, translated by the unpack
     unsigned small_cap;        // shared-memory path: ring slots (power of two)
 };
 
@@ -113,6 +122,17 @@ cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm);
 cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int32_t *hub_base,
                               int2 **chunk_tab_out, int64_t *n_chunks_out, cudaStream_t s);
 cudaError_t launch_queue_reset(const tq_device_view &q, unsigned long long t0, cudaStream_t s);
+
+// relabel.cu: degree-descending vertex relabelling of a CSR (plan build).
+// Nothing is allocated (out stays zero) unless the largest degree exceeds
+// min_max_degree; the caller then owns out's four pool buffers.
+struct RelabelOut {
+    int32_t *new2old, *old2new;
+    int64_t *row_ptr;
+    int32_t *col;
+};
+cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int min_max_degree,
+                          RelabelOut *out, cudaStream_t s);
 
 // bfs_small.cu: the whole run (load, BFS over a shared-memory queue, unpack)
 // in one 1024-thread block, for graphs whose state fits in shared memory

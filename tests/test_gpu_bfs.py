@@ -593,3 +593,62 @@ def test_persisting_l2_limit_is_reference_counted(tq):
     b.run(r, lv, None)
     b.close()
     assert limit() == before
+
+
+@pytest.mark.parametrize("parents", ["any", "min_id"])
+@pytest.mark.parametrize("relabel", [-1, 1])
+def test_relabelled_plans(tq, relabel, parents):
+    """bfs_opts.relabel: the plan runs on a
+    degree-sorted copy of the CSR, but roots, outputs and parent ids are in
+    the original numbering -- levels identical to the oracle, min-id parents
+    identical (the minimum over ORIGINAL ids), 'any' parents Graph500-valid;
+    roots include the top hub and an isolated vertex; a uniform grid and a
+    tree (relabelled only when forced) too; host-CSR plans as well."""
+    import torch
+    graphs = [kronecker_csr(13, 16, 3), grid_csr(64, 40), tree4_csr(20000)]
+    for g in graphs:
+        rp, col = to_dev(g)
+        deg = g.degrees()
+        roots = [int(np.argmax(deg)), int(sample_roots(g.row_ptr, 1, 4)[0]), g.n_vertices - 1]
+        if (deg == 0).any():
+            roots.append(int(np.flatnonzero(deg == 0)[0]))
+        lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+        pa = torch.empty_like(lv)
+        with tq.BfsPlan(rp, col, parents=parents, relabel=relabel, smem_path=-1, timeout_s=20) as plan:
+            for r in roots:
+                st = plan.run(r, lv, pa)
+                check_against_oracle(g, r, lv, pa, st, min_id=parents == "min_id")
+                assert st["relabelled"] == (relabel > 0)
+            lvb = np.empty(len(roots) * g.n_vertices, dtype=np.int32)
+            pab = np.empty_like(lvb)
+            stats = plan.run_batch(roots, lvb, pab)
+            for i, r in enumerate(roots):
+                n = g.n_vertices
+                check_against_oracle(g, r, lvb[i * n:(i + 1) * n], pab[i * n:(i + 1) * n], stats[i],
+                                     min_id=parents == "min_id")
+    g = kronecker_csr(12, 16, 8)
+    r = int(sample_roots(g.row_ptr, 1, 1)[0])
+    lh, ph, st = tq.bfs(g.row_ptr, g.col, r, parents=parents, relabel=relabel, smem_path=-1)  # host CSR
+    check_against_oracle(g, r, lh, ph, st, min_id=parents == "min_id")
+    assert st["relabelled"] == (relabel > 0)
+
+
+def test_relabel_auto_rule(tq):
+    """Auto: a graph with a vertex of more than `chunk` edges (Kronecker) is
+    relabelled, a uniform grid is not; delay injection and chunk tokens on a
+    relabelled plan stay exact."""
+    g = kronecker_csr(14, 16, 2)
+    rp, col = to_dev(g)
+    r = int(sample_roots(g.row_ptr, 1, 3)[0])
+    level, parent, st = tq.bfs(rp, col, r)
+    check_against_oracle(g, r, level, parent, st)
+    assert st["relabelled"] == 1 and st["chunk_tasks"] > 0
+    for seed in range(3):
+        level, parent, st = tq.bfs(rp, col, r, parents="min_id", chunk=64, debug_delay_ns=20000,
+                                   debug_delay_seed=seed)
+        check_against_oracle(g, r, level, parent, st, min_id=True)
+    gg = grid_csr(256, 256)
+    rp, col = to_dev(gg)
+    level, parent, st = tq.bfs(rp, col, 0)
+    check_against_oracle(gg, 0, level, parent, st)
+    assert st["relabelled"] == 0
