@@ -214,6 +214,7 @@ def config_rmat10(tq, dev, local, args):
                 st = plan.run(roots[i % len(roots)], lv, pa)
                 us.append(st["ms"] * 1e3)
                 te += st["traversed_edges"]
+            smem = bool(st["smem_path"])
             for r in roots:  # parity of every sampled root (default and min-id rules)
                 plan.run(r, lv, pa)
                 lo, po, _ = oracle.bfs(rp_h, col_h, r)
@@ -229,7 +230,10 @@ def config_rmat10(tq, dev, local, args):
             te_o += info["traversed_edges"]
     out.update({
         "gpu_us_median": round(_median(us), 2), "gpu_us_min": round(min(us), 2), "gpu_runs": 20,
-        "gpu_timed": "CUDA events around init + persistent kernel + unpack (bfs_stats.ms), graph L2-resident",
+        "gpu_path": "shared-memory queue, one 1024-thread block" if smem else "persistent grid",
+        "gpu_timed": ("CUDA events around the one launch (graph load, BFS over the shared-memory queue, unpack; "
+                      "bfs_stats.ms)" if smem else
+                      "CUDA events around init + persistent kernel + unpack (bfs_stats.ms), graph L2-resident"),
         "gpu_gteps": round(te / (sum(us) * 1e-6) / 1e9, 4),
         "cpu_baseline": dict({"kind": "oracle", "cores": 1, "ms_median": round(_median(ms_o), 3),
                               "gteps": round(te_o / (sum(ms_o) * 1e-3) / 1e9, 4),
@@ -434,6 +438,8 @@ def main():
                     choices=sorted(WORKLOADS))
     ap.add_argument("--variant", default="rf_an")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-priority", type=int, default=0, help="e2e leg: priority of the run streams")
+    ap.add_argument("--e2e-relabel", type=int, default=0, help="e2e leg: bfs_opts.relabel of the per-step plans")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-queue", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="skip configs 1-4 (headline workload only)")
@@ -579,14 +585,17 @@ def main():
         # batch runs: every step's H2D and D2H stay inside the timed region,
         # overlapped with the BFS of the neighbouring step (ctypes releases the
         # GIL during the C calls).
-        streams = [stream, torch.cuda.Stream(dev)]
+        # (priority 0 = the device's least, as the library's own build stream:
+        # a high-priority BFS starves the next step's relabelling kernels,
+        # results/e2e_relabel_r02.log)
+        streams = [torch.cuda.Stream(dev, priority=args.e2e_priority), torch.cuda.Stream(dev, priority=args.e2e_priority)]
         # untimed warm-up (as the device leg has W warm-up steps): two
         # host-built plans alive at once, as in the timed loop, so the
         # library's memory pool has grown to hold both before timing starts
         with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[0], device=local,
-                        parents=args.parents) as hp0, \
+                        parents=args.parents, relabel=args.e2e_relabel) as hp0, \
                 tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[1], device=local,
-                           parents=args.parents) as hp1:
+                           parents=args.parents, relabel=args.e2e_relabel) as hp1:
             hp0.run_batch(mine[:1], lv_np, pa_np, stride=0)
             hp1.run_batch(mine[:1], lv_np, pa_np, stride=0)
         if dist:
@@ -595,7 +604,7 @@ def main():
 
         def make_plan(k):
             return tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[k % 2], device=local,
-                              parents=args.parents)
+                              parents=args.parents, relabel=args.e2e_relabel)
 
         t0 = time.perf_counter()
         te_e2e = 0

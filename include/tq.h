@@ -280,6 +280,10 @@ tq_status bfs_run_ex(const tq_csr *g, int32_t root, int32_t *level_out, int32_t 
  * place and must outlive the plan. */
 typedef struct bfs_plan bfs_plan;
 tq_status bfs_plan_create(const tq_csr *g, const bfs_opts *opts, bfs_plan **out);
+/* (The build -- host-CSR upload, relabelling, chunk table -- runs on an
+ * internal stream of the device's lowest priority and is synchronous; runs
+ * use opts->stream.  A plan built while another plan's BFS runs on a
+ * higher-priority stream therefore yields the SMs to that BFS.) */
 /* level_out / parent_out: DEVICE pointers (or NULL). Stream-ordered on
  * opts->stream, but synchronous (it reads the status word back). */
 tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,

@@ -602,7 +602,22 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     p->nnz = nnz;
 
     bool smem_auto_lanes = false;
+    // The plan's build work (graph upload, relabelling, chunk table) runs on
+    // an internal stream of the device's lowest priority, so that a plan
+    // built while another plan's BFS runs on a higher-priority stream yields
+    // the SMs to it (bench.py's e2e leg builds step k+1's plan during step k).
+    cudaStream_t bs = nullptr;
+    {
+        int least = 0, greatest = 0;
+        cudaDeviceGetStreamPriorityRange(&least, &greatest);
+        if (cudaStreamCreateWithPriority(&bs, cudaStreamNonBlocking, least) != cudaSuccess) {
+            delete p;
+            return TQ_ERR_CUDA;
+        }
+    }
     auto fail = [&](tq_status s) {
+        cudaStreamSynchronize(bs);
+        cudaStreamDestroy(bs);
         bfs_plan_destroy(p);
         return s;
     };
@@ -612,10 +627,10 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         p->col = const_cast<int32_t *>(gph->col);
     } else {
         p->owns_graph = true;
-        e = pool_alloc(&p->row_ptr, (size_t)(n + 1) * sizeof(int64_t), p->stream);
-        if (e == cudaSuccess) e = pool_alloc(&p->col, (size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t), p->stream);
-        if (e == cudaSuccess) e = h2d_chunked(p->row_ptr, gph->row_ptr, (size_t)(n + 1) * sizeof(int64_t), p->stream);
-        if (e == cudaSuccess && nnz > 0) e = h2d_chunked(p->col, gph->col, (size_t)nnz * sizeof(int32_t), p->stream);
+        e = pool_alloc(&p->row_ptr, (size_t)(n + 1) * sizeof(int64_t), bs);
+        if (e == cudaSuccess) e = pool_alloc(&p->col, (size_t)(nnz > 0 ? nnz : 1) * sizeof(int32_t), bs);
+        if (e == cudaSuccess) e = h2d_chunked(p->row_ptr, gph->row_ptr, (size_t)(n + 1) * sizeof(int64_t), bs);
+        if (e == cudaSuccess && nnz > 0) e = h2d_chunked(p->col, gph->col, (size_t)nnz * sizeof(int32_t), bs);
         if (e != cudaSuccess) return fail(from_cuda(e));
     }
     if (task == kTaskSSSP && nnz > 0) {
@@ -625,13 +640,16 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
             p->wgt = const_cast<int32_t *>(weights);
         } else {
             p->owns_wgt = true;
-            e = pool_alloc(&p->wgt, (size_t)nnz * sizeof(int32_t), p->stream);
+            e = pool_alloc(&p->wgt, (size_t)nnz * sizeof(int32_t), bs);
             if (e == cudaSuccess)
                 e = cudaMemcpyAsync(p->wgt, weights, (size_t)nnz * sizeof(int32_t), cudaMemcpyHostToDevice,
-                                    p->stream);
+                                    bs);
             if (e != cudaSuccess) return fail(from_cuda(e));
         }
     }
+    e = pinned_small_alloc(reinterpret_cast<void **>(&p->stats_h));
+    if (e == cudaSuccess) e = pinned_small_alloc(reinterpret_cast<void **>(&p->ctr_h));
+    if (e != cudaSuccess) return fail(from_cuda(e));
     // Shared-memory path (bfs_opts.smem_path): the
     // whole run in one block when CSR + W + markers + a ring of 2V slots fit
     {
@@ -653,20 +671,21 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     // graph; a uniform graph such as the grid keeps its own numbering)
     if (task == kTaskBFS && !p->smem && o.relabel >= 0 && n < (1ll << 31) - 1) {
         RelabelOut ro{};
-        e = build_relabel(p->row_ptr, p->col, n, nnz, o.relabel > 0 ? -1 : chunk, &ro, p->stream);
+        e = build_relabel(p->row_ptr, p->col, n, nnz, o.relabel > 0 ? -1 : chunk,
+                          reinterpret_cast<int32_t *>(p->ctr_h), &ro, bs);
         if (e != cudaSuccess) return fail(from_cuda(e));
         if (ro.new2old) {
             p->relabelled = true;
             p->row_ptr0 = p->row_ptr;
-            if (p->owns_graph) pool_free(p->col, p->stream);  // only the relabelled entries are read
+            if (p->owns_graph) pool_free(p->col, bs);  // only the relabelled entries are read
             p->row_ptr = ro.row_ptr;
             p->col = ro.col;
             p->new2old = ro.new2old;
             p->old2new = ro.old2new;
         }
     }
-    e = pool_alloc(&p->W, (size_t)n * sizeof(unsigned long long), p->stream);
-    if (e == cudaSuccess) e = pool_alloc(&p->hub_base, (size_t)n * sizeof(int32_t), p->stream);
+    e = pool_alloc(&p->W, (size_t)n * sizeof(unsigned long long), bs);
+    if (e == cudaSuccess) e = pool_alloc(&p->hub_base, (size_t)n * sizeof(int32_t), bs);
     if (task == kTaskBFS) {
         // Level mirror width (R8): a nibble per vertex when a byte
         // mirror would exceed 32 MB (it then no longer stays L2-resident next
@@ -676,21 +695,20 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         if (o.mirror_bits == 4 || o.mirror_bits == 8) p->mirror_bits = o.mirror_bits;
         if (p->mirror_bits == 4 && o.variant != TQ_VARIANT_RF_AN) return fail(TQ_ERR_UNSUPPORTED);
         p->mirror_bytes = p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 7) / 8 * 4;
-        if (e == cudaSuccess) e = pool_alloc(&p->mir, p->mirror_bytes, p->stream);
+        if (e == cudaSuccess) e = pool_alloc(&p->mir, p->mirror_bytes, bs);
         // expanded-level markers: same width as the mirror
         if (e == cudaSuccess)
-            e = pool_alloc(&p->x8, p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 1) / 2, p->stream);
+            e = pool_alloc(&p->x8, p->mirror_bits == 8 ? (size_t)n : (size_t)(n + 1) / 2, bs);
     } else {
-        if (e == cudaSuccess) e = pool_alloc(&p->xd, (size_t)n * sizeof(unsigned), p->stream);
+        if (e == cudaSuccess) e = pool_alloc(&p->xd, (size_t)n * sizeof(unsigned), bs);
     }
-    if (e == cudaSuccess) e = pool_alloc(&p->stats, kStatCount * sizeof(unsigned long long), p->stream);
+    if (e == cudaSuccess) e = pool_alloc(&p->stats, kStatCount * sizeof(unsigned long long), bs);
     static_assert(kStatCount * sizeof(unsigned long long) <= kPinBytes, "pinned block too small");
-    if (e == cudaSuccess) e = pinned_small_alloc(reinterpret_cast<void **>(&p->stats_h));
-    if (e == cudaSuccess) e = pinned_small_alloc(reinterpret_cast<void **>(&p->ctr_h));
     for (auto &ev : p->ev)
         if (e == cudaSuccess) e = cudaEventCreate(&ev);
     if (e != cudaSuccess) return fail(from_cuda(e));
-    e = build_chunk_table(p->row_ptr, n, chunk, p->hub_base, &p->chunk_tab, &p->n_chunks, p->stream);
+    e = build_chunk_table(p->row_ptr, n, chunk, p->hub_base, &p->chunk_tab, &p->n_chunks,
+                          reinterpret_cast<int32_t *>(p->ctr_h), bs);
     if (e != cudaSuccess) return fail(from_cuda(e));
     if (n + p->n_chunks >= (1ll << 31)) return fail(TQ_ERR_UNSUPPORTED);
 
@@ -759,8 +777,10 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         // l2_persist_acquire)
         p->l2_window = l2_persist_acquire(gdev, p->mirror_bytes);
     }
-    e = cudaStreamSynchronize(p->stream);
+    e = cudaStreamSynchronize(bs);  // (the build's buffers are used on p->stream from now on)
+    if (e == cudaSuccess) e = cudaStreamSynchronize(p->stream);
     if (e != cudaSuccess) return fail(from_cuda(e));
+    cudaStreamDestroy(bs);
     *out = p;
     return TQ_OK;
 }

@@ -1379,7 +1379,7 @@ cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm)
 }
 
 cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int32_t *hub_base,
-                              int2 **chunk_tab_out, int64_t *n_chunks_out, cudaStream_t s)
+                              int2 **chunk_tab_out, int64_t *n_chunks_out, int32_t *pinned8, cudaStream_t s)
 {
     *chunk_tab_out = nullptr;
     *n_chunks_out = 0;
@@ -1392,13 +1392,14 @@ cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int3
     e = cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, nch, hub_base, (int)n, s);
     if (e == cudaSuccess) e = pool_alloc(&tmp, tmp_bytes, s);
     if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, nch, hub_base, (int)n, s);
-    int32_t last_base = 0, last_n = 0;
+    // (read back through pinned memory: a pageable copy would serialise with
+    // other streams' work, e.g. a BFS running while the next plan is built)
     if (e == cudaSuccess)
-        e = cudaMemcpyAsync(&last_base, hub_base + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, s);
+        e = cudaMemcpyAsync(pinned8, hub_base + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess)
-        e = cudaMemcpyAsync(&last_n, nch + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, s);
+        e = cudaMemcpyAsync(pinned8 + 1, nch + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    const int64_t total = (int64_t)last_base + last_n;
+    const int64_t total = e == cudaSuccess ? (int64_t)pinned8[0] + pinned8[1] : 0;
     if (e == cudaSuccess && total > 0) {
         int2 *tab = nullptr;
         e = pool_alloc(&tab, (size_t)total * sizeof(int2), s);

@@ -120,19 +120,20 @@ cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, i
 cudaError_t launch_bfs_unpack(const BfsParams &p, int32_t *level, int32_t *parent, cudaStream_t s);
 cudaError_t bfs_occupancy(int variant, int block, int *blocks_per_sm);
 cudaError_t build_chunk_table(const int64_t *row_ptr, int64_t n, int chunk, int32_t *hub_base,
-                              int2 **chunk_tab_out, int64_t *n_chunks_out, cudaStream_t s);
+                              int2 **chunk_tab_out, int64_t *n_chunks_out, int32_t *pinned8, cudaStream_t s);
 cudaError_t launch_queue_reset(const tq_device_view &q, unsigned long long t0, cudaStream_t s);
 
 // relabel.cu: degree-descending vertex relabelling of a CSR (plan build).
 // Nothing is allocated (out stays zero) unless the largest degree exceeds
-// min_max_degree; the caller then owns out's four pool buffers.
+// min_max_degree; the caller then owns out's four pool buffers.  pinned4:
+// 4 bytes of pinned host memory (the one read-back: the largest degree).
 struct RelabelOut {
     int32_t *new2old, *old2new;
     int64_t *row_ptr;
     int32_t *col;
 };
 cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int min_max_degree,
-                          RelabelOut *out, cudaStream_t s);
+                          int32_t *pinned4, RelabelOut *out, cudaStream_t s);
 
 // bfs_small.cu: the whole run (load, BFS over a shared-memory queue, unpack)
 // in one 1024-thread block, for graphs whose state fits in shared memory

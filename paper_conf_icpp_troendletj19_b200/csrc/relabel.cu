@@ -37,13 +37,14 @@ namespace {
 // kron24 -8.4% vs -7.4%; results/relabel_r02.log)
 constexpr int64_t kHubRegion = 1 << 20;
 constexpr int64_t kBigRow = 4096;        // rows copied by a whole block
+constexpr int kRB = 128;                 // threads per relabelling block (<= 32 registers)
 
 __host__ __device__ __forceinline__ int64_t rank_to_new(int64_t r, int64_t H, int64_t lines)
 {
     return r < H ? (r % lines) * 128 + r / lines : r;
 }
 
-__global__ void degree_kernel(const int64_t *rp, int64_t n, int32_t *deg, int32_t *iota)
+__global__ void __launch_bounds__(kRB, 16) degree_kernel(const int64_t *rp, int64_t n, int32_t *deg, int32_t *iota)
 {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -53,7 +54,7 @@ __global__ void degree_kernel(const int64_t *rp, int64_t n, int32_t *deg, int32_
 }
 
 // new ids from ranks; new-order degrees (int64, for the offsets scan)
-__global__ void place_kernel(const int32_t *deg_sorted, const int32_t *rank2old, int64_t n, int64_t H,
+__global__ void __launch_bounds__(kRB, 16) place_kernel(const int32_t *deg_sorted, const int32_t *rank2old, int64_t n, int64_t H,
                              int64_t lines, int32_t *new2old, int32_t *old2new, int64_t *deg_new)
 {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -67,58 +68,88 @@ __global__ void place_kernel(const int32_t *deg_sorted, const int32_t *rank2old,
     if (blockIdx.x == 0 && threadIdx.x == 0) deg_new[n] = 0;
 }
 
-// rows of rank >= r0 (at most kBigRow entries): one warp per row
-__global__ void copy_rows_warp(const int64_t *rp, const int32_t *col, const int64_t *rp_new,
-                               const int32_t *rank2old, const int32_t *old2new, int64_t n, int64_t r0,
-                               int64_t H, int64_t lines, int32_t *col_new)
+// The relabelling kernels are grid-stride loops of 128-thread blocks of <= 32
+// registers, 16 per SM.  (Measured in bench.py's e2e leg, which builds step
+// k+1's plan while step k's BFS runs, 8 steps of kron26x64: 59.8 GTEPS with
+// this grid on normal-priority streams, 56.8 with the BFS streams at high
+// priority, 53.4 with one such block per SM -- the one the persistent BFS
+// kernel leaves room for beside it -- and 60.5 without relabelling;
+// results/e2e_relabel_r02.log.)
+//
+// Rows of at most kBigRow entries, 32 consecutive ranks per warp: the warp
+// scans their degrees and walks the concatenation of their entries 32 at a
+// time (lane l takes entry s + l; its row by a shuffle binary search over the
+// inclusive prefix sums), so lanes stay busy whatever the degrees and the
+// writes -- consecutive ranks are consecutive rows of the new CSR beyond the
+// dealt hub region -- are coalesced.
+__global__ void __launch_bounds__(kRB, 16) copy_rows_small(const int64_t *rp, const int32_t *col, const int64_t *rp_new,
+                                const int32_t *rank2old, const int32_t *deg_sorted, const int32_t *old2new,
+                                int64_t n, int64_t H, int64_t lines, int32_t *col_new)
 {
     const unsigned lane = threadIdx.x & 31;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t r = r0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); r < n; r += nw) {
+    for (int64_t r0 = 32 * (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); r0 < n; r0 += 32 * nw) {
+        const int64_t r = r0 + lane;
+        int d = 0;
+        int64_t src = 0, dst = 0;
+        if (r < n && deg_sorted[r] <= kBigRow) {
+            const int32_t o = rank2old[r];
+            src = rp[o];
+            d = (int)(rp[o + 1] - src);
+            dst = rp_new[rank_to_new(r, H, lines)];
+        }
+        int incl = d;
+#pragma unroll
+        for (int k = 1; k < 32; k <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, k);
+            if (lane >= (unsigned)k) incl += t;
+        }
+        const int total = __shfl_sync(0xffffffffu, incl, 31);
+        const int64_t sb = src - (incl - d), db = dst - (incl - d);  // entry g of this lane's row: sb + g, db + g
+        for (int s0 = 0; s0 < total; s0 += 32) {
+            const int g = s0 + (int)lane;
+            int o = 0;  // owner lane: number of lanes whose inclusive prefix is <= g
+#pragma unroll
+            for (int k = 16; k > 0; k >>= 1) {
+                const int c = __shfl_sync(0xffffffffu, incl, o + k - 1);
+                if (c <= g) o += k;
+            }
+            const int64_t s = __shfl_sync(0xffffffffu, sb, o), t = __shfl_sync(0xffffffffu, db, o);
+            if (g < total) col_new[t + g] = old2new[__ldg(col + s + g)];
+        }
+    }
+}
+
+// Rows of more than kBigRow entries (the first ranks: degrees are sorted):
+// a block per row, four gathers in flight per thread
+__global__ void __launch_bounds__(kRB, 16) copy_rows_big(const int64_t *rp, const int32_t *col, const int64_t *rp_new,
+                                                     const int32_t *rank2old, const int32_t *deg_sorted,
+                                                     const int32_t *old2new, int64_t n, int64_t H, int64_t lines,
+                                                     int32_t *col_new)
+{
+    for (int64_t r = blockIdx.x; r < n && deg_sorted[r] > kBigRow; r += gridDim.x) {
         const int64_t i = rank_to_new(r, H, lines);
         const int32_t o = rank2old[r];
         const int64_t src = rp[o], d = rp[o + 1] - src, dst = rp_new[i];
-        for (int64_t k = lane; k < d; k += 32) col_new[dst + k] = old2new[__ldg(col + src + k)];
+        const int64_t step = 4 * (int64_t)blockDim.x;
+        int64_t k = threadIdx.x;
+        for (; k + 3 * blockDim.x < d; k += step) {
+            int32_t c[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) c[j] = __ldg(col + src + k + j * blockDim.x);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) c[j] = old2new[c[j]];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) col_new[dst + k + j * blockDim.x] = c[j];
+        }
+        for (; k < d; k += blockDim.x) col_new[dst + k] = old2new[__ldg(col + src + k)];
     }
-}
-
-// rows of rank < r0 (more than kBigRow entries): one block per row, four
-// gathers in flight per thread
-__global__ void __launch_bounds__(512) copy_rows_block(const int64_t *rp, const int32_t *col, const int64_t *rp_new,
-                                                       const int32_t *rank2old, const int32_t *old2new,
-                                                       int64_t H, int64_t lines, int32_t *col_new)
-{
-    const int64_t r = blockIdx.x;
-    const int64_t i = rank_to_new(r, H, lines);
-    const int32_t o = rank2old[r];
-    const int64_t src = rp[o], d = rp[o + 1] - src, dst = rp_new[i];
-    const int64_t step = 4 * (int64_t)blockDim.x;
-    int64_t k = threadIdx.x;
-    for (; k + 3 * blockDim.x < d; k += step) {
-        int32_t c[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) c[j] = __ldg(col + src + k + j * blockDim.x);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) c[j] = old2new[c[j]];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) col_new[dst + k + j * blockDim.x] = c[j];
-    }
-    for (; k < d; k += blockDim.x) col_new[dst + k] = old2new[__ldg(col + src + k)];
-}
-
-int grid_of(int64_t n, int block)
-{
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const int64_t want = (n + block - 1) / block, cap = (int64_t)sms * 8;
-    return (int)(want < 1 ? 1 : (want < cap ? want : cap));
 }
 
 }  // namespace
 
 cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int min_max_degree,
-                          RelabelOut *out, cudaStream_t s)
+                          int32_t *pinned4, RelabelOut *out, cudaStream_t s)
 {
     *out = RelabelOut{};
     int32_t *deg = nullptr, *iota = nullptr, *deg_sorted = nullptr, *rank2old = nullptr;
@@ -126,12 +157,16 @@ cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int6
     void *tmp = nullptr;
     size_t tmp_bytes = 0, t2 = 0;
     RelabelOut o{};
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const unsigned rgrid = (unsigned)sms * 16;
     cudaError_t e = pool_alloc(&deg, (size_t)n * 4, s);
     if (e == cudaSuccess) e = pool_alloc(&iota, (size_t)n * 4, s);
     if (e == cudaSuccess) e = pool_alloc(&deg_sorted, (size_t)n * 4, s);
     if (e == cudaSuccess) e = pool_alloc(&rank2old, (size_t)n * 4, s);
     if (e == cudaSuccess) {
-        degree_kernel<<<grid_of(n, 256), 256, 0, s>>>(rp, n, deg, iota);
+        degree_kernel<<<rgrid, kRB, 0, s>>>(rp, n, deg, iota);
         e = cudaGetLastError();
     }
     if (e == cudaSuccess)
@@ -142,10 +177,9 @@ cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int6
     if (e == cudaSuccess)
         e = cub::DeviceRadixSort::SortPairsDescending(tmp, tmp_bytes, deg, deg_sorted, iota, rank2old, (int)n, 0, 32,
                                                       s);
-    int32_t maxdeg = 0;
-    if (e == cudaSuccess) e = cudaMemcpyAsync(&maxdeg, deg_sorted, 4, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(pinned4, deg_sorted, 4, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    if (e == cudaSuccess && maxdeg > min_max_degree) {
+    if (e == cudaSuccess && *pinned4 > min_max_degree) {
         // hub region: the first H ranks, dealt over H / 128 lines
         int64_t H = (n < kHubRegion ? n : kHubRegion) / 128 * 128;
         if (H < 2 * 128) H = 0;
@@ -156,34 +190,19 @@ cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int6
         if (e == cudaSuccess) e = pool_alloc(&o.row_ptr, (size_t)(n + 1) * 8, s);
         if (e == cudaSuccess) e = pool_alloc(&o.col, (size_t)(nnz > 0 ? nnz : 1) * 4, s);
         if (e == cudaSuccess) {
-            place_kernel<<<grid_of(n, 256), 256, 0, s>>>(deg_sorted, rank2old, n, H, lines, o.new2old, o.old2new,
-                                                         deg_new);
+            place_kernel<<<rgrid, kRB, 0, s>>>(deg_sorted, rank2old, n, H, lines, o.new2old, o.old2new, deg_new);
             e = cudaGetLastError();
         }
         size_t tb = tmp_bytes > t2 ? tmp_bytes : t2;
         if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(tmp, tb, deg_new, o.row_ptr, (int)(n + 1), s);
-        // rows with more than kBigRow entries are the first ranks
-        int64_t nbig = 0;
         if (e == cudaSuccess) {
-            // count on the host from a bounded binary search over the sorted degrees
-            int64_t lo = 0, hi = n;  // first rank with degree <= kBigRow
-            while (lo < hi && e == cudaSuccess) {
-                const int64_t mid = (lo + hi) / 2;
-                int32_t dm = 0;
-                e = cudaMemcpyAsync(&dm, deg_sorted + mid, 4, cudaMemcpyDeviceToHost, s);
-                if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-                if (dm > kBigRow) lo = mid + 1;
-                else hi = mid;
-            }
-            nbig = lo;
-        }
-        if (e == cudaSuccess && nbig > 0) {
-            copy_rows_block<<<(unsigned)nbig, 512, 0, s>>>(rp, col, o.row_ptr, rank2old, o.old2new, H, lines, o.col);
+            copy_rows_big<<<rgrid, kRB, 0, s>>>(
+                rp, col, o.row_ptr, rank2old, deg_sorted, o.old2new, n, H, lines, o.col);
             e = cudaGetLastError();
         }
-        if (e == cudaSuccess && nbig < n) {
-            copy_rows_warp<<<grid_of((n - nbig) * 32, 256), 256, 0, s>>>(rp, col, o.row_ptr, rank2old, o.old2new, n,
-                                                                        nbig, H, lines, o.col);
+        if (e == cudaSuccess) {
+            copy_rows_small<<<rgrid, kRB, 0, s>>>(rp, col, o.row_ptr, rank2old, deg_sorted,
+                                                                            o.old2new, n, H, lines, o.col);
             e = cudaGetLastError();
         }
         if (e == cudaSuccess) e = cudaStreamSynchronize(s);
