@@ -230,6 +230,11 @@ typedef struct {
                            numbering (min-id parents too).  0 = auto (default):
                            on when some vertex has more than `chunk` edges;
                            < 0 = off; > 0 = on                              */
+    int level_bits;     /* TEST ONLY: width cap of the level field that RF/AN
+                           BFS tokens carry (R22) -- levels at or
+                           beyond 2^level_bits - 1 then travel the fenced
+                           path; 0 = every bit the ids leave (default);
+                           1..30                                            */
 } bfs_opts;
 
 enum { TQ_PARENT_ANY = 0, TQ_PARENT_MIN_ID = 1 };
@@ -259,6 +264,10 @@ typedef struct {
     int32_t ticket_lanes;       /* lanes per warp holding main-queue tickets      */
     int32_t smem_path;          /* 1: the run used the shared-memory path         */
     int32_t relabelled;         /* 1: the plan runs on a relabelled copy (opts)   */
+    int32_t level_tokens;       /* 1: the run's tokens carried their levels
+                                   (R22; a plan whose levels outgrew
+                                   the token's level field runs later BFS with
+                                   acquire polls instead)                       */
 } bfs_stats;
 
 /* Single-source BFS.  level_out[v] = hop distance from root (-1 unreached);

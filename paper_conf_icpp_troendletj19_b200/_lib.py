@@ -44,7 +44,7 @@ class bfs_opts(ctypes.Structure):
                 ("debug_delay_ns", ctypes.c_int), ("debug_delay_seed", c_u32),
                 ("cas_backoff_ns", ctypes.c_int), ("mirror_bits", ctypes.c_int), ("deep_grid", ctypes.c_int),
                 ("ticket_lanes", ctypes.c_int), ("l2_persist", ctypes.c_int),
-                ("smem_path", ctypes.c_int), ("relabel", ctypes.c_int)]
+                ("smem_path", ctypes.c_int), ("relabel", ctypes.c_int), ("level_bits", ctypes.c_int)]
 
 
 class bfs_stats(ctypes.Structure):
@@ -55,7 +55,7 @@ class bfs_stats(ctypes.Structure):
                 ("busy_cycles", c_u64), ("rounds", c_u64), ("skipped_tasks", c_u64),
                 ("max_level", c_i32), ("persistent_threads", c_i32), ("mirror_bits", c_i32),
                 ("ticket_lanes", c_i32), ("smem_path", c_i32),
-                ("relabelled", c_i32)]
+                ("relabelled", c_i32), ("level_tokens", c_i32)]
 
 
 class tq_bench_cfg(ctypes.Structure):

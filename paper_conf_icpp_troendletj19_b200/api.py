@@ -76,7 +76,7 @@ def _csr(row_ptr, col) -> _lib.tq_csr:
 def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None, timeout_s=0.0,
           backoff_ns=0, device=0, parents="any", hub_queue=True, debug_delay_ns=0,
           debug_delay_seed=0, cas_backoff_ns=0, mirror_bits=0, deep_grid=True, ticket_lanes=0,
-          l2_persist=True, smem_path=0, relabel=0) -> _lib.bfs_opts:
+          l2_persist=True, smem_path=0, relabel=0, level_bits=0) -> _lib.bfs_opts:
     return _lib.bfs_opts(int(capacity), int(threads), int(block), int(chunk), _variant(variant),
                          stream, float(timeout_s), int(backoff_ns), int(device),
                          _lib.PARENT_RULES[parents] if isinstance(parents, str) else int(parents),
@@ -84,13 +84,14 @@ def _opts(variant="rf_an", capacity=0, threads=0, block=0, chunk=0, stream=None,
                          int(cas_backoff_ns), int(mirror_bits), 0 if deep_grid else -1, int(ticket_lanes),
                          0 if l2_persist else -1,
                          int(smem_path) if not isinstance(smem_path, bool) else (1 if smem_path else -1),
-                         int(relabel) if not isinstance(relabel, bool) else (1 if relabel else -1))
+                         int(relabel) if not isinstance(relabel, bool) else (1 if relabel else -1),
+                         int(level_bits))
 
 
 # bfs / BfsPlan keyword options that map one to one onto bfs_opts fields
 _OPT_KEYS = ("variant", "capacity", "threads", "chunk", "timeout_s", "backoff_ns", "parents", "hub_queue",
              "debug_delay_ns", "debug_delay_seed", "cas_backoff_ns", "mirror_bits", "deep_grid", "ticket_lanes",
-             "l2_persist", "smem_path", "relabel")
+             "l2_persist", "smem_path", "relabel", "level_bits")
 
 
 def _stats_dict(st: _lib.bfs_stats) -> dict:
@@ -114,7 +115,7 @@ def bfs(row_ptr, col, root: int, level=None, parent=None, *, want_parent: bool =
     chunk, timeout_s, backoff_ns, parents, hub_queue, debug_delay_ns,
     debug_delay_seed, cas_backoff_ns, mirror_bits, deep_grid, ticket_lanes, l2_persist,
     smem_path: 0 auto, -1 / False off, 1 / True required; relabel: 0 auto, -1 / False off,
-    1 / True on).
+    1 / True on; level_bits: test-only cap of the tokens' level field).
     """
     bad = set(opts) - set(_OPT_KEYS)
     if bad:

@@ -337,6 +337,9 @@ struct bfs_plan {
     // vertex relabelling (relabel.cu): row_ptr / col are then the plan-owned
     // relabelled CSR and row_ptr0 the original offsets (owned if owns_graph)
     bool relabelled = false;
+    bool lit = true;                          // BFS tokens carry their level (bfs.cu, R22)
+    int level_bits = 0;                       // test-only cap of the level field (bfs_opts.level_bits)
+    unsigned lit_field = 0;                   // the largest level both token kinds can carry
     int32_t *new2old = nullptr, *old2new = nullptr;
     int64_t *row_ptr0 = nullptr;
     unsigned smem_cap = 0;                    // its ring slots
@@ -595,6 +598,11 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
         return TQ_ERR_INVALID;
     }
     p->cas_backoff_ns = o.cas_backoff_ns;
+    if (o.level_bits < 0 || o.level_bits > 30) {
+        delete p;
+        return TQ_ERR_INVALID;
+    }
+    p->level_bits = o.level_bits;
     p->delay_ns = o.debug_delay_ns;
     p->delay_seed = o.debug_delay_seed;
     p->task = task;
@@ -854,6 +862,17 @@ static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t 
     bp.old2new = p->old2new;
     bp.row_ptr0 = p->row_ptr0;
     bp.pid_orig = p->relabelled && p->parent_rule == TQ_PARENT_MIN_ID;
+    // token layout: as few id bits as the ids need, the rest carry the level
+    bp.tok_vbits = 1;
+    while (bp.tok_vbits < 31 && (1ll << bp.tok_vbits) < p->n) ++bp.tok_vbits;
+    bp.tok_cbits = 1;
+    while (bp.tok_cbits < 31 && (1ll << bp.tok_cbits) < p->n_chunks) ++bp.tok_cbits;
+    if (p->level_bits > 0) {  // test: a narrower level field (more id bits)
+        if (bp.tok_vbits < 31u - p->level_bits) bp.tok_vbits = 31u - p->level_bits;
+        if (bp.tok_cbits < 31u - p->level_bits) bp.tok_cbits = 31u - p->level_bits;
+    }
+    bp.lit = p->lit ? 1 : 0;
+    p->lit_field = 0x7FFFFFFFu >> (bp.tok_vbits > bp.tok_cbits ? bp.tok_vbits : bp.tok_cbits);
     if (p->smem) {
         // one launch: graph load, BFS over the shared-memory queue, unpack
         // (its statistics and status land where the grid path puts them;
@@ -932,6 +951,7 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
         stats->ticket_lanes = p->ticket_lanes;
         stats->smem_path = p->smem ? 1 : 0;
         stats->relabelled = p->relabelled ? 1 : 0;
+        stats->level_tokens = (!p->smem && p->task == kTaskBFS && p->variant == TQ_VARIANT_RF_AN && p->lit) ? 1 : 0;
         if (p->smem) stats->persistent_threads = 1024;
     }
     // Deep graphs: a BFS of >= 1,024 levels runs a few thousand
@@ -939,6 +959,11 @@ static tq_status plan_finish(bfs_plan *p, bfs_stats *stats)
     // idle polls of its 189K held tickets (the paper's too-many-threads
     // dilemma).  After such a run the plan (same graph) launches one
     // block per SM: grid 4096^2 53 -> ~46 ms.  Only when threads == 0.
+    // Levels in the tokens (R22): a run whose levels did not fit the field
+    // published its deeper tokens with a release fence and took them with an
+    // acquire re-read, dearer than the plain acquire polls; the plan's later
+    // runs (same graph) use the acquire polls throughout.
+    if (status == TQ_FINISHED && p->stats_h[ST_MAX_LEVEL] >= p->lit_field) p->lit = false;
     if (p->auto_blocks && status == TQ_FINISHED && p->stats_h[ST_MAX_LEVEL] >= 1024) {
         const int deep_blocks = sm_count(p->device);
         if (p->blocks > deep_blocks) p->blocks = deep_blocks;

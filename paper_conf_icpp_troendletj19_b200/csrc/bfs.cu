@@ -377,7 +377,8 @@ __device__ __forceinline__ bool an_reserve_rear(const tq_device_view &q, unsigne
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const uint32_t *items,
                                                unsigned cnt, unsigned lane, unsigned *qatom,
-                                               unsigned *casfail, unsigned long long lap_end, unsigned bo_max)
+                                               unsigned *casfail, unsigned long long lap_end, unsigned bo_max,
+                                               bool need_fence = true)
 {
     if (cnt == 0) return;
     if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_AN) {
@@ -392,8 +393,9 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
                 ++*qatom;
             }
             // release: the W updates (and this warp's Rear reservation) are
-            // ordered before the tokens that name them
-            tq_fence_release();
+            // ordered before the tokens that name them -- needed only when a
+            // token does not carry its level (R22)
+            if (need_fence) tq_fence_release();
             base = tq_shfl64(b0, 0);
         } else {
             if (!an_reserve_rear(q, cnt, &base, qatom, casfail, bo_max)) return;
@@ -444,11 +446,22 @@ __device__ __forceinline__ void enqueue_staged(const tq_device_view &q, const ui
     }
 }
 
+// LIT (R22): does any of the cnt staged vertex tokens lack its
+// level (all-ones level field)?  Then the flush needs the release fence.
+__device__ __forceinline__ bool staged_unknown(const uint32_t *items, unsigned cnt, unsigned lane, unsigned vb)
+{
+    const unsigned lu = 0x7FFFFFFFu >> vb;
+    bool u = false;
+    for (unsigned i = lane; i < cnt; i += 32) u |= (items[i] >> vb) == lu;
+    return __any_sync(TQ_FULL_MASK, u);
+}
+
 // chunk tokens of one hub: CHUNK_FLAG | (first + k), k < n (warp-uniform args)
 template <int VARIANT>
 __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t first, unsigned n,
                                                unsigned lane, unsigned *qatom, unsigned *casfail,
-                                               unsigned long long lap_end, unsigned bo_max)
+                                               unsigned long long lap_end, unsigned bo_max,
+                                               uint32_t lvbits = 0, bool need_fence = true)
 {
     if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY) {
         for (unsigned i = lane; i < n; i += 32)
@@ -462,9 +475,9 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
                 b0 = tq_atom_add(q.rear, (unsigned long long)n);
                 ++*qatom;
             }
-            // release: a chunk token names the hub's W entry (its level), and
-            // this warp's Rear reservation is ordered before its Done increment
-            tq_fence_release();
+            // release: a chunk token names the hub's W entry (its level) --
+            // needed only when the token does not carry the level (R22)
+            if (need_fence) tq_fence_release();
             base = tq_shfl64(b0, 0);
         } else if constexpr (VARIANT == TQ_VARIANT_AN) {
             if (!an_reserve_rear(q, n, &base, qatom, casfail, bo_max)) return;
@@ -483,17 +496,17 @@ __device__ __forceinline__ void enqueue_chunks(const tq_device_view &q, uint32_t
         if (VARIANT == TQ_VARIANT_RF_AN && base + n <= lap_end) {  // first lap: no full check
             for (unsigned i = lane; i < n; i += 32)
                 tq_st_relaxed(q.slots + ((base + i) & q.mask),
-                              ((unsigned long long)(CHUNK_FLAG | (first + i)) << 32) | (unsigned)(base + i + 1));
+                              ((unsigned long long)(CHUNK_FLAG | lvbits | (first + i)) << 32) | (unsigned)(base + i + 1));
             return;
         }
-        for (unsigned i = lane; i < n; i += 32) tq_publish(q, base + i, CHUNK_FLAG | (first + i));
+        for (unsigned i = lane; i < n; i += 32) tq_publish(q, base + i, CHUNK_FLAG | lvbits | (first + i));
     }
 }
 
 // ---------------------------------------------------------------------------
 // The persistent kernel
 // ---------------------------------------------------------------------------
-template <int VARIANT, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, int MIR = 8>
+template <int VARIANT, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, int MIR = 8, bool LITT = false>
 __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsParams p)
 {
     constexpr unsigned kMirSat = Mirror<MIR>::kSat;
@@ -532,6 +545,21 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
     unsigned st_qatom = 0, st_fail = 0;
     const bool min_id = p.parent_rule == TQ_PARENT_MIN_ID;
     unsigned backoff = 0, idle = 0, busy = 0;
+    // Level in the token (R22; RF/AN BFS): a vertex token is
+    // [0 | level : 31 - vb | id : vb], a chunk token [1 | level : 31 - cb | id : cb]
+    // (vb, cb = p.tok_vbits, p.tok_cbits); an all-ones level field means
+    // "not carried" (the level did not fit).  A consumer of a token that
+    // carries its level needs nothing its producer wrote besides the slot
+    // word, so such tokens are published without a release fence and
+    // polled without acquire semantics (no L1 invalidation per poll).
+    // (an instantiation of its own: a plan whose levels outgrew the field
+    // runs the kernel without it, unchanged)
+    constexpr bool LIT = LITT && VARIANT == TQ_VARIANT_RF_AN && TASK == kTaskBFS;
+    // LIT: tasks finished, added to Done when the warp goes idle (lane 0; in
+    // shared memory, out of the hot loop's registers)
+    __shared__ unsigned pend_done_all[kWarps];
+    unsigned &pend_done = pend_done_all[threadIdx.x >> 5];
+    if (lane == 0) pend_done = 0;
 
     // Listing 1, split in two halves: the proxy's
     // atomic_add(Front, n) for the lanes that became hungry is issued right
@@ -600,9 +628,13 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             // lane issues both polls back to back and prefers the chunk
             // (acquire loads: a hit makes the producer's W update visible,
             // with no fence; ld.acquire.gpu is LDG.STRONG.GPU + CCTL.IVALL)
-            const unsigned long long sv0 = have ? tq_ld_acquire(q.slots + (tk & q.mask)) : 0ull;
+            // (LIT: relaxed; the rare token without its level takes a fence below)
+            const unsigned long long sv0 =
+                have ? (LIT ? tq_ld_relaxed(q.slots + (tk & q.mask)) : tq_ld_acquire(q.slots + (tk & q.mask))) : 0ull;
             const unsigned long long sv1 =
-                (q1_lane && have1) ? tq_ld_acquire(q1.slots + (tk1 & q1.mask)) : 0ull;
+                (q1_lane && have1) ? (LIT ? tq_ld_relaxed(q1.slots + (tk1 & q1.mask))
+                                          : tq_ld_acquire(q1.slots + (tk1 & q1.mask)))
+                                   : 0ull;
             got1 = q1_lane && have1 && (unsigned)sv1 == tk1 + 1u;
             got = !got1 && have && (unsigned)sv0 == tk + 1u;
             item = (uint32_t)((got1 ? sv1 : sv0) >> 32);
@@ -625,6 +657,15 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         if (gm == 0) {
             // ---- idle work cycle: Algorithm 1 line 1, WorkRemains() ----
             if (lane == 0) ++S[ST_EMPTY_POLLS];
+            if constexpr (LIT) {
+                // Done += the tasks this warp finished (R6), released
+                // after every Rear reservation of theirs (all issued by lane 0)
+                if (lane == 0 && pend_done) {
+                    tq_fence_release();
+                    tq_red_add_relaxed(q.done, (unsigned long long)pend_done);
+                    pend_done = 0;
+                }
+            }
             ++idle;
             if ((idle & 3) == 0 && tq_status_read(q, warp_gid) != TQ_RUNNING) break;
             // termination test: 1 warp in 8, every 4 idle cycles, so idle
@@ -661,6 +702,25 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         }
         if constexpr (VARIANT == TQ_VARIANT_CAS_RETRY || VARIANT == TQ_VARIANT_AN)
             tq_fence_gpu();  // acquire for the comparators' relaxed dequeues
+        // LIT: the token's level field; a token without one was published
+        // after a release fence, and its consumer acquires before reading W
+        bool unk = false;
+        unsigned Lt = 0;
+        if constexpr (LIT) {
+            if (got) {
+                const unsigned b = (item & CHUNK_FLAG) ? p.tok_cbits : p.tok_vbits;
+                Lt = (item & ~CHUNK_FLAG) >> b;
+                unk = Lt == (0x7FFFFFFFu >> b);
+                // its producer fenced before publishing it: an acquire re-read
+                // of the (still full) slot synchronises with that release
+                if (unk) {
+                    if (got1)
+                        tq_ld_acquire(q1.slots + (tk1 & q1.mask));
+                    else
+                        tq_ld_acquire(q.slots + (tk & q.mask));
+                }
+            }
+        }
         if constexpr (VARIANT == TQ_VARIANT_RF_AN || VARIANT == TQ_VARIANT_PER_THREAD_AFA) {
             if (got0) {  // put the slot back to dna for the next lap
                 tq_st_relaxed(q.slots + (tk & q.mask), (unsigned long long)(tk + cap32));
@@ -696,13 +756,13 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
         bool skipped = false;
         if (got) {
             if (item & CHUNK_FLAG) {
-                const int2 c = p.chunk_tab[item & ~CHUNK_FLAG];
+                const int2 c = p.chunk_tab[LIT ? (item & ((1u << p.tok_cbits) - 1u)) : (item & ~CHUNK_FLAG)];
                 v = c.x;
                 const long long re = ld_nc_i64(p.row_ptr + v + 1);
                 lo = ld_nc_i64(p.row_ptr + v) + (long long)c.y * chunk;
                 hi = min(lo + (long long)chunk, re);
             } else {
-                v = (int32_t)item;
+                v = (int32_t)(LIT ? (item & ((1u << p.tok_vbits) - 1u)) : item);
                 lo = ld_nc_i64(p.row_ptr + v);
                 hi = ld_nc_i64(p.row_ptr + v + 1);
                 if (hi - lo > chunk) {  // hub: schedule its sub-tasks instead
@@ -722,7 +782,12 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             // original numbering); else v itself (the unpack translates)
             const unsigned pid = (TASK == kTaskBFS && p.pid_orig) ? (unsigned)__ldg(p.new2old + v) : (unsigned)v;
             // current cost of the node (Listing 2 line 21), read fresh
-            const unsigned L = (unsigned)(tq_ld_relaxed(p.W + v) >> 32);
+            // (LIT: the token's level, or a lower one W already holds: any
+            // value read is a level v has held, so the relaxed read is safe)
+            unsigned L = (unsigned)(tq_ld_relaxed(p.W + v) >> 32);
+            if constexpr (LIT) {
+                if (!unk) L = min(L, Lt);
+            }
             if (dly == 1) __nanosleep(p.delay_ns);
             if constexpr (TASK == kTaskSSSP) {
                 // the edge weight is added per edge in the expansion
@@ -958,7 +1023,14 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         }
                         n_reenq += __popc(__ballot_sync(TQ_FULL_MASK, nt && oldhi != 0xffffffffu));
                         const unsigned m = __ballot_sync(TQ_FULL_MASK, nt);
-                        if (nt) stage[wr + __popc(m & tq_lanemask_lt())] = cv;
+                        if (nt) {
+                            uint32_t tok = cv;
+                            if constexpr (LIT) {  // the token carries its level (R22)
+                                const unsigned lu = 0x7FFFFFFFu >> p.tok_vbits;
+                                tok |= min(L1, lu) << p.tok_vbits;
+                            }
+                            stage[wr + __popc(m & tq_lanemask_lt())] = tok;
+                        }
                         wr += __popc(m);
                         __syncwarp();
                     }
@@ -999,7 +1071,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             }
             if (cnt > kStageCap - 32 * KU) {
                 __syncwarp();
-                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end, p.cas_backoff_ns);
+                enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end, p.cas_backoff_ns,
+                                        !LIT || staged_unknown(stage, cnt, lane, p.tok_vbits));
                 __syncwarp();
                 cnt = 0;
             }
@@ -1007,7 +1080,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
 
         // ---- ScheduleNewlyDiscoveredWorkTokens(): Listing 3 ----
         __syncwarp();
-        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end, p.cas_backoff_ns);
+        enqueue_staged<VARIANT>(q, stage, cnt, lane, &st_qatom, &st_fail, p.q_lap_end, p.cas_backoff_ns,
+                                !LIT || staged_unknown(stage, cnt, lane, p.tok_vbits));
         __syncwarp();
         unsigned hubm = __ballot_sync(TQ_FULL_MASK, nch > 0);
         while (hubm) {
@@ -1015,8 +1089,16 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             hubm &= hubm - 1;
             const unsigned n = __shfl_sync(TQ_FULL_MASK, nch, h);
             const uint32_t first = __shfl_sync(TQ_FULL_MASK, chb, h);
+            uint32_t lvbits = 0;
+            bool fence = true;
+            if constexpr (LIT) {  // the chunk tokens carry the hub's level
+                const unsigned Lh = __shfl_sync(TQ_FULL_MASK, (unsigned)(offer >> 32) - 1u, h);
+                const unsigned lu = 0x7FFFFFFFu >> p.tok_cbits;
+                lvbits = min(Lh, lu) << p.tok_cbits;
+                fence = Lh >= lu;
+            }
             enqueue_chunks<VARIANT>(hubq ? q1 : q, first, n, lane, &st_qatom, &st_fail,
-                                    hubq ? p.q1_lap_end : p.q_lap_end, p.cas_backoff_ns);
+                                    hubq ? p.q1_lap_end : p.q_lap_end, p.cas_backoff_ns, lvbits, fence);
         }
 
         // ---- completion accounting for WorkRemains() (R6) ----
@@ -1028,8 +1110,12 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
             // release fence that follows each reservation (staged tokens and
             // chunk tokens alike) already ordered it before this increment.
             if (lane == 0) {
-                tq_red_add_relaxed(q.done, (unsigned long long)__popc(gm));
-                ++st_qatom;
+                if constexpr (LIT) {
+                    pend_done += __popc(gm);  // added when the warp goes idle
+                } else {
+                    tq_red_add_relaxed(q.done, (unsigned long long)__popc(gm));
+                    ++st_qatom;
+                }
             }
         } else {
             __syncwarp();
@@ -1315,7 +1401,7 @@ cudaError_t launch_queue_reset(const tq_device_view &q, unsigned long long t0, c
     return cudaGetLastError();
 }
 
-template <int V, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, int MIR = 8>
+template <int V, int TASK = kTaskBFS, int KU = kU, int MINB = kMinBlocks, int MIR = 8, bool LITT = false>
 static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStream_t s)
 {
     if (block != kBlock) return cudaErrorInvalidValue;
@@ -1337,7 +1423,7 @@ static cudaError_t launch_v(const BfsParams &p, int blocks, int block, cudaStrea
         cfg.attrs = attr;
         cfg.numAttrs = 1;
     }
-    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, TASK, KU, MINB, MIR>, p);
+    return cudaLaunchKernelEx(&cfg, bfs_persistent_kernel<V, TASK, KU, MINB, MIR, LITT>, p);
 }
 
 cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, int block,
@@ -1348,9 +1434,12 @@ cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, i
         return launch_v<TQ_VARIANT_RF_AN, kTaskSSSP>(p, blocks, block, s);
     }
     switch (variant) {
-    case TQ_VARIANT_RF_AN:
-        if (p.mirror_bits == 4) return launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 4>(p, blocks, block, s);
-        return launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
+    case TQ_VARIANT_RF_AN:  // with / without levels in the tokens (R22)
+        if (p.mirror_bits == 4)
+            return p.lit ? launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 4, true>(p, blocks, block, s)
+                         : launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 4>(p, blocks, block, s);
+        return p.lit ? launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 8, true>(p, blocks, block, s)
+                     : launch_v<TQ_VARIANT_RF_AN>(p, blocks, block, s);
     case TQ_VARIANT_PER_THREAD_AFA: return launch_v<TQ_VARIANT_PER_THREAD_AFA>(p, blocks, block, s);
     case TQ_VARIANT_CAS_RETRY: return launch_v<TQ_VARIANT_CAS_RETRY>(p, blocks, block, s);
     case TQ_VARIANT_AN: return launch_v<TQ_VARIANT_AN>(p, blocks, block, s);

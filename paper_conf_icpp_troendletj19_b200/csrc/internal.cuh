@@ -106,6 +106,11 @@ struct BfsParams {
     const int32_t *new2old;
     const int32_t *old2new;
     const int64_t *row_ptr0;   // the original row offsets (unpack statistics)
+    // RF/AN BFS token layout (R22): id bits of vertex / chunk tokens;
+    // the bits between them and the chunk flag carry the token's level
+    unsigned tok_vbits;
+    unsigned tok_cbits;
+    int lit;                   // levels travel in the tokens (off once a plan's levels outgrew the field)
     int pid_orig;              // W's parent field holds original ids (relabelled
                                // min-id plans: the kernel reads new2old); else
                                // the plan's own ids, translated by the unpack

@@ -652,3 +652,41 @@ def test_relabel_auto_rule(tq):
     level, parent, st = tq.bfs(rp, col, 0)
     check_against_oracle(gg, 0, level, parent, st)
     assert st["relabelled"] == 0
+
+
+@pytest.mark.parametrize("parents", ["any", "min_id"])
+@pytest.mark.parametrize("level_bits", [0, 1, 2, 3])
+def test_level_tokens(tq, level_bits, parents):
+    """RF/AN BFS tokens carry their level (R22): a consumer then
+    needs no acquire and a producer no release fence.  Levels that do not fit
+    the field travel the fenced path (producer fence, consumer acquire
+    re-read of the slot); a plan whose levels outgrew the field runs its later
+    BFS with acquire polls.  bfs_opts.level_bits (test only) narrows the field
+    so that both kinds of token mix within one run, also under delay injection
+    (stale W reads) and with hub chunk tokens."""
+    import torch
+    graphs = [kronecker_csr(13, 16, 3), grid_csr(70, 41), tree4_csr(20000)]
+    for g in graphs:
+        rp, col = to_dev(g)
+        lv = torch.empty(g.n_vertices, dtype=torch.int32, device="cuda")
+        pa = torch.empty_like(lv)
+        roots = [int(r) for r in sample_roots(g.row_ptr, 3, 7)]
+        with tq.BfsPlan(rp, col, parents=parents, level_bits=level_bits, chunk=64, smem_path=-1,
+                        timeout_s=20) as plan:
+            sts = []
+            for r in roots:
+                st = plan.run(r, lv, pa)
+                check_against_oracle(g, r, lv, pa, st, min_id=parents == "min_id")
+                sts.append(st)
+            field = (1 << level_bits) - 1 if level_bits else None
+            assert sts[0]["level_tokens"] == 1
+            if field is not None and sts[0]["max_level"] >= field:
+                assert sts[1]["level_tokens"] == 0  # outgrown: acquire polls from then on
+            if level_bits == 0:
+                assert all(s["level_tokens"] == 1 for s in sts)
+        with tq.BfsPlan(rp, col, parents=parents, level_bits=level_bits, chunk=64, smem_path=-1, timeout_s=20,
+                        debug_delay_ns=20000, debug_delay_seed=level_bits) as plan:
+            st = plan.run(roots[0], lv, pa)
+            check_against_oracle(g, roots[0], lv, pa, st, min_id=parents == "min_id")
+    with pytest.raises(tq.TQError):
+        tq.bfs(rp, col, 0, level_bits=31)
