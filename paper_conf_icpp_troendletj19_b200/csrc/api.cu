@@ -679,7 +679,13 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     // graph; a uniform graph such as the grid keeps its own numbering)
     if (task == kTaskBFS && !p->smem && o.relabel >= 0 && n < (1ll << 31) - 1) {
         RelabelOut ro{};
-        e = build_relabel(p->row_ptr, p->col, n, nnz, o.relabel > 0 ? -1 : chunk,
+        // hub region (ranks dealt over their lines): 2^14 where the byte
+        // mirror's probes are L1-cached (bfs.cu), so the top hubs' bytes stay
+        // within the L1; 2^20 for the nibble mirror (results/relabel_r02.log,
+        // results/level_tokens_r02.log)
+        const bool byte_mirror = !(p->variant == TQ_VARIANT_RF_AN && n > (1ll << 25)) || o.mirror_bits == 8;
+        const int64_t hub_region = (byte_mirror && o.mirror_bits != 4) ? (1ll << 14) : (1ll << 20);
+        e = build_relabel(p->row_ptr, p->col, n, nnz, o.relabel > 0 ? -1 : chunk, hub_region,
                           reinterpret_cast<int32_t *>(p->ctr_h), &ro, bs);
         if (e != cudaSuccess) return fail(from_cuda(e));
         if (ro.new2old) {

@@ -113,6 +113,16 @@ __device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long lon
     asm volatile("ld.global.cg.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
+// The byte mirror's probe through L1 (a weak load): stale-high values are all
+// the prefilter needs (R8), and with levels in the tokens (R22) no acquire
+// poll invalidates the L1, so the relabelled plan's top hubs (the first 2^14
+// ids, relabel.cu) stay cached there.  kron24: -3.5% (results/level_tokens_r02.log).
+__device__ __forceinline__ unsigned ld_l1_u8(const uint8_t *p, unsigned long long pol)
+{
+    unsigned v;
+    asm("ld.global.L2::cache_hint.u8 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
 __device__ __forceinline__ unsigned mix32(unsigned x)
 {
     x ^= x >> 16;
@@ -942,7 +952,9 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                     // deep graphs, e.g. the grid's 8,191 levels), go to atomicMin
                     const bool deep = lv1[j] >= kMirSat;
                     if constexpr (MIR == 8)
-                        b8[j] = (val[j] && !deep) ? ld_cg_u8((const uint8_t *)p.mir + u[j], pol_keep) : 0xFFu;
+                        b8[j] = (val[j] && !deep) ? (LIT ? ld_l1_u8((const uint8_t *)p.mir + u[j], pol_keep)
+                                                          : ld_cg_u8((const uint8_t *)p.mir + u[j], pol_keep))
+                                                  : 0xFFu;
                     else
                         b8[j] = (val[j] && !deep) ? ld_cg_u32(p.mir + ((unsigned)u[j] >> 3), pol_keep) : ~0u;
                 }

@@ -138,7 +138,7 @@ struct RelabelOut {
     int32_t *col;
 };
 cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int min_max_degree,
-                          int32_t *pinned4, RelabelOut *out, cudaStream_t s);
+                          int64_t hub_region, int32_t *pinned4, RelabelOut *out, cudaStream_t s);
 
 // bfs_small.cu: the whole run (load, BFS over a shared-memory queue, unpack)
 // in one 1024-thread block, for graphs whose state fits in shared memory

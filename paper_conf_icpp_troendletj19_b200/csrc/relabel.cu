@@ -8,7 +8,7 @@
 // W words, markers and row offsets each sit in their own 32-byte sector.  The
 // plan therefore renumbers vertices by descending degree (stable, so equal
 // degrees keep their order), which packs the hubs' per-vertex state into few
-// sectors; the first kHubRegion ranks are dealt round-robin over the region's
+// sectors; the first hub_region ranks are dealt round-robin over the region's
 // 128-byte lines (rank r -> (r mod lines) * 128 + r / lines) so that the very
 // top hubs -- the most-probed bytes -- land in different lines and L2 slices
 // instead of all in the first one.  Measured (results/relabel_r02.log): kron24
@@ -33,9 +33,7 @@ namespace tqk {
 
 namespace {
 
-// ranks dealt over the region's lines: 2^20 (kron26 -6.2% vs -2.2% with 2^17,
-// kron24 -8.4% vs -7.4%; results/relabel_r02.log)
-constexpr int64_t kHubRegion = 1 << 20;
+
 constexpr int64_t kBigRow = 4096;        // rows copied by a whole block
 constexpr int kRB = 128;                 // threads per relabelling block (<= 32 registers)
 
@@ -149,7 +147,7 @@ __global__ void __launch_bounds__(kRB, 16) copy_rows_big(const int64_t *rp, cons
 }  // namespace
 
 cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int min_max_degree,
-                          int32_t *pinned4, RelabelOut *out, cudaStream_t s)
+                          int64_t hub_region, int32_t *pinned4, RelabelOut *out, cudaStream_t s)
 {
     *out = RelabelOut{};
     int32_t *deg = nullptr, *iota = nullptr, *deg_sorted = nullptr, *rank2old = nullptr;
@@ -181,7 +179,7 @@ cudaError_t build_relabel(const int64_t *rp, const int32_t *col, int64_t n, int6
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess && *pinned4 > min_max_degree) {
         // hub region: the first H ranks, dealt over H / 128 lines
-        int64_t H = (n < kHubRegion ? n : kHubRegion) / 128 * 128;
+        int64_t H = (n < hub_region ? n : hub_region) / 128 * 128;
         if (H < 2 * 128) H = 0;
         const int64_t lines = H ? H / 128 : 1;
         e = pool_alloc(&o.new2old, (size_t)n * 4, s);
