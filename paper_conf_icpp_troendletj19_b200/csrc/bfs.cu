@@ -831,7 +831,8 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         hi = lo;
                         nch = 0;
                     } else {
-                        st_u8(p.x8 + v, L < kLvlSat ? L : kLvlSat);
+                        // (a saturated marker never skips: not stored)
+                        if (L < kLvlSat) st_u8(p.x8 + v, L);
                     }
                 } else {
                     const unsigned xb = ld_relaxed_u8(p.x8 + ((unsigned)v >> 1));
@@ -1026,7 +1027,11 @@ __global__ void __launch_bounds__(kBlock, MINB) bfs_persistent_kernel(const BfsP
                         // it the same way, so a missed lowering costs one
                         // extra atomicMin, not one per later probe.
                         if constexpr (MIR == 8) {
-                            if (nt) st_u8((uint8_t *)p.mir + cv, L1 < kMirSat ? L1 : kMirSat);
+                            // (a saturated entry filters nothing -- offers at
+                            // or past saturation skip the probe -- so it is not
+                            // stored: on deep graphs the flush's release fence
+                            // then has no store of this round to wait for)
+                            if (nt && L1 < kMirSat) st_u8((uint8_t *)p.mir + cv, L1);
                         } else {
                             const unsigned nv = nt ? L1 : oldhi;  // v's level now
                             const unsigned sh = (cv & 7u) << 2;
