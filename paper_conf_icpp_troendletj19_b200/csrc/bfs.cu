@@ -1450,8 +1450,23 @@ cudaError_t launch_bfs_persistent(int variant, const BfsParams &p, int blocks, i
         if (variant != TQ_VARIANT_RF_AN) return cudaErrorInvalidValue;
         return launch_v<TQ_VARIANT_RF_AN, kTaskSSSP>(p, blocks, block, s);
     }
+    // One block per SM (small graphs, deep-graph plans): the instantiation
+    // compiled for one resident block, with every register it wants instead
+    // of the 48 that five blocks allow (grid 4096^2: 41.0 -> 38.7 ms,
+    // results/deep_stores_r02.log)
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const bool one_per_sm = blocks <= sms;
     switch (variant) {
     case TQ_VARIANT_RF_AN:  // with / without levels in the tokens (R22)
+        if (one_per_sm) {
+            if (p.mirror_bits == 4)
+                return p.lit ? launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, 1, 4, true>(p, blocks, block, s)
+                             : launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, 1, 4>(p, blocks, block, s);
+            return p.lit ? launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, 1, 8, true>(p, blocks, block, s)
+                         : launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, 1, 8>(p, blocks, block, s);
+        }
         if (p.mirror_bits == 4)
             return p.lit ? launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 4, true>(p, blocks, block, s)
                          : launch_v<TQ_VARIANT_RF_AN, kTaskBFS, kU, kMinBlocks, 4>(p, blocks, block, s);
