@@ -439,7 +439,9 @@ def main():
     ap.add_argument("--variant", default="rf_an")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-priority", type=int, default=0, help="e2e leg: priority of the run streams")
-    ap.add_argument("--e2e-relabel", type=int, default=0, help="e2e leg: bfs_opts.relabel of the per-step plans")
+    ap.add_argument("--e2e-relabel", type=int, default=-1,
+                    help="e2e leg: bfs_opts.relabel of the per-step plans (default off: a plan rebuilt every "
+                         "step for 64 roots does not win its relabelling back, results/e2e_relabel_r02.log)")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-queue", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="skip configs 1-4 (headline workload only)")

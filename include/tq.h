@@ -289,10 +289,11 @@ tq_status bfs_run_ex(const tq_csr *g, int32_t root, int32_t *level_out, int32_t 
  * place and must outlive the plan. */
 typedef struct bfs_plan bfs_plan;
 tq_status bfs_plan_create(const tq_csr *g, const bfs_opts *opts, bfs_plan **out);
-/* (The build -- host-CSR upload, relabelling, chunk table -- runs on an
- * internal stream of the device's lowest priority and is synchronous; runs
- * use opts->stream.  A plan built while another plan's BFS runs on a
- * higher-priority stream therefore yields the SMs to that BFS.) */
+/* (The build -- host-CSR upload, chunk table -- runs on an internal stream
+ * and is synchronous; runs use opts->stream.  A plan's vertex relabelling
+ * (bfs_opts.relabel) is done by its first run, on opts->stream, before the
+ * BFS: that first launch is then synchronous, and a plan built while another
+ * plan's BFS runs does not relabel beside it.) */
 /* level_out / parent_out: DEVICE pointers (or NULL). Stream-ordered on
  * opts->stream, but synchronous (it reads the status word back). */
 tq_status bfs_plan_run(bfs_plan *p, int32_t root, int32_t *level_out, int32_t *parent_out,

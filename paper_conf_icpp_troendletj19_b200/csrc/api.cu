@@ -337,6 +337,9 @@ struct bfs_plan {
     // vertex relabelling (relabel.cu): row_ptr / col are then the plan-owned
     // relabelled CSR and row_ptr0 the original offsets (owned if owns_graph)
     bool relabelled = false;
+    bool relabel_pending = false;             // relabel at the first run (plan_relabel)
+    int relabel_min_deg = 0;
+    int64_t hub_region = 0;
     bool lit = true;                          // BFS tokens carry their level (bfs.cu, R22)
     int level_bits = 0;                       // test-only cap of the level field (bfs_opts.level_bits)
     unsigned lit_field = 0;                   // the largest level both token kinds can carry
@@ -676,27 +679,20 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     }
     // Vertex relabelling (bfs_opts.relabel, relabel.cu): BFS on the persistent
     // grid, auto when a vertex has more than `chunk` edges (a degree-skewed
-    // graph; a uniform graph such as the grid keeps its own numbering)
+    // graph; a uniform graph such as the grid keeps its own numbering).  Done
+    // at the plan's first run, on its own stream (plan_relabel): a plan built
+    // while another plan's BFS runs -- bench.py's e2e leg builds step k+1's
+    // plan during step k -- would otherwise relabel beside that BFS and slow
+    // it far more than the relabelling's own ~25 ms (results/e2e_relabel_r02.log).
     if (task == kTaskBFS && !p->smem && o.relabel >= 0 && n < (1ll << 31) - 1) {
-        RelabelOut ro{};
+        p->relabel_pending = true;
+        p->relabel_min_deg = o.relabel > 0 ? -1 : chunk;
         // hub region (ranks dealt over their lines): 2^14 where the byte
         // mirror's probes are L1-cached (bfs.cu), so the top hubs' bytes stay
         // within the L1; 2^20 for the nibble mirror (results/relabel_r02.log,
         // results/level_tokens_r02.log)
         const bool byte_mirror = !(p->variant == TQ_VARIANT_RF_AN && n > (1ll << 25)) || o.mirror_bits == 8;
-        const int64_t hub_region = (byte_mirror && o.mirror_bits != 4) ? (1ll << 14) : (1ll << 20);
-        e = build_relabel(p->row_ptr, p->col, n, nnz, o.relabel > 0 ? -1 : chunk, hub_region,
-                          reinterpret_cast<int32_t *>(p->ctr_h), &ro, bs);
-        if (e != cudaSuccess) return fail(from_cuda(e));
-        if (ro.new2old) {
-            p->relabelled = true;
-            p->row_ptr0 = p->row_ptr;
-            if (p->owns_graph) pool_free(p->col, bs);  // only the relabelled entries are read
-            p->row_ptr = ro.row_ptr;
-            p->col = ro.col;
-            p->new2old = ro.new2old;
-            p->old2new = ro.old2new;
-        }
+        p->hub_region = (byte_mirror && o.mirror_bits != 4) ? (1ll << 14) : (1ll << 20);
     }
     e = pool_alloc(&p->W, (size_t)n * sizeof(unsigned long long), bs);
     if (e == cudaSuccess) e = pool_alloc(&p->hub_base, (size_t)n * sizeof(int32_t), bs);
@@ -810,12 +806,44 @@ tq_status sssp_plan_create(const tq_csr *gph, const int32_t *weights, const bfs_
     return plan_create_impl(gph, weights, kTaskSSSP, opts, out);
 }
 
+// The plan's vertex relabelling (relabel.cu), at its first
+// run, on its stream (synchronous).  The chunk table names vertices, so it
+// is rebuilt on the new numbering (same chunk count).
+static tq_status plan_relabel(bfs_plan *p)
+{
+    p->relabel_pending = false;
+    RelabelOut ro{};
+    cudaStream_t s = p->stream;
+    cudaError_t e = build_relabel(p->row_ptr, p->col, p->n, p->nnz, p->relabel_min_deg, p->hub_region,
+                                  reinterpret_cast<int32_t *>(p->ctr_h), &ro, s);
+    if (e != cudaSuccess) return from_cuda(e);
+    if (!ro.new2old) return TQ_OK;  // no vertex above the degree threshold
+    p->relabelled = true;
+    p->row_ptr0 = p->row_ptr;
+    if (p->owns_graph) pool_free(p->col, s);  // only the relabelled entries are read
+    p->row_ptr = ro.row_ptr;
+    p->col = ro.col;
+    p->new2old = ro.new2old;
+    p->old2new = ro.old2new;
+    pool_free(p->chunk_tab, s);
+    p->chunk_tab = nullptr;
+    int64_t nch = 0;
+    e = build_chunk_table(p->row_ptr, p->n, p->chunk, p->hub_base, &p->chunk_tab, &nch,
+                          reinterpret_cast<int32_t *>(p->ctr_h), s);
+    if (e != cudaSuccess) return from_cuda(e);
+    return nch == p->n_chunks ? TQ_OK : TQ_ERR_CUDA;
+}
+
 // First half of a run: enqueue init + persistent kernel + unpack and the
 // status / statistics read-back on the plan's stream; returns immediately.
 static tq_status plan_launch(bfs_plan *p, int32_t root, int32_t *level, int32_t *parent)
 {
     cudaStream_t s = p->stream;
     if (p->in_flight) return TQ_ERR_INVALID;
+    if (p->relabel_pending) {
+        tq_status st = plan_relabel(p);
+        if (st != TQ_OK) return st;
+    }
     if (p->dirty) {
         tq_status st = tq_reset(p->q, s);
         if (st == TQ_OK && p->q1) st = tq_reset(p->q1, s);
