@@ -652,6 +652,16 @@ def test_relabel_auto_rule(tq):
     level, parent, st = tq.bfs(rp, col, 0)
     check_against_oracle(gg, 0, level, parent, st)
     assert st["relabelled"] == 0
+    # the relabelling happens at a plan's first run, whichever entry point it is
+    roots = [int(x) for x in sample_roots(g.row_ptr, 3, 11)]
+    lvb = np.empty(3 * g.n_vertices, dtype=np.int32)
+    pab = np.empty_like(lvb)
+    with tq.BfsPlan(g.row_ptr, g.col) as plan:  # host CSR: the plan owns its copies
+        stats = plan.run_batch(roots, lvb, pab)
+    n = g.n_vertices
+    for i, r in enumerate(roots):
+        check_against_oracle(g, r, lvb[i * n:(i + 1) * n], pab[i * n:(i + 1) * n], stats[i])
+        assert stats[i]["relabelled"] == 1
 
 
 @pytest.mark.parametrize("parents", ["any", "min_id"])
