@@ -30,7 +30,32 @@ for v in ("rf_an", "per_thread_afa", "cas_retry", "an"):
                 plan.run(r, lv, pa)
                 lo, _, _ = oracle.bfs(g.row_ptr, g.col, r, parents=False)
                 assert np.array_equal(lv.cpu().numpy(), lo), (v, parents, r)
-with tq.BfsPlan(rp, col, capacity=64, threads=4096, timeout_s=60) as plan:
+# round 2, session 3 paths: the shared-memory single-block BFS (and its
+# queue-full abort), the persistent grid with level-carrying tokens, a
+# relabelled plan with hub chunks, and a narrow level field (fenced tokens mixed in)
+for sp in (1, -1):
+    for parents in ("any", "min_id"):
+        with tq.BfsPlan(rp, col, parents=parents, smem_path=sp, threads=4096, timeout_s=60) as plan:
+            for r in roots:
+                plan.run(r, lv, pa)
+                lo, _, _ = oracle.bfs(g.row_ptr, g.col, r, parents=False)
+                assert np.array_equal(lv.cpu().numpy(), lo), ("smem", sp, parents, r)
+try:
+    tq.bfs(rp, col, int(np.argmax(g.degrees())), capacity=64, smem_path=1)
+    raise SystemExit("expected a queue-full abort on the shared-memory path")
+except tq.TQError as e:
+    assert e.status == -4
+g2 = kronecker_csr(12, 16, 3)
+rp2, col2 = torch.from_numpy(g2.row_ptr).cuda(), torch.from_numpy(g2.col).cuda()
+lv2 = torch.empty(g2.n_vertices, dtype=torch.int32, device="cuda")
+pa2 = torch.empty_like(lv2)
+for kw in ({"relabel": 1, "chunk": 32}, {"relabel": 1, "level_bits": 2, "parents": "min_id"}):
+    with tq.BfsPlan(rp2, col2, threads=4096, timeout_s=60, **kw) as plan:
+        for r in [int(x) for x in sample_roots(g2.row_ptr, 2, 4)]:
+            plan.run(r, lv2, pa2)
+            lo, _, _ = oracle.bfs(g2.row_ptr, g2.col, r, parents=False)
+            assert np.array_equal(lv2.cpu().numpy(), lo), (kw, r)
+with tq.BfsPlan(rp, col, capacity=64, threads=4096, timeout_s=60, smem_path=-1) as plan:
     try:
         plan.run(int(np.argmax(g.degrees())), lv, pa)
         raise SystemExit("expected a queue-full abort")
