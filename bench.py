@@ -591,52 +591,51 @@ def main():
         # a high-priority BFS starves the next step's relabelling kernels,
         # results/e2e_relabel_r02.log)
         streams = [torch.cuda.Stream(dev, priority=args.e2e_priority), torch.cuda.Stream(dev, priority=args.e2e_priority)]
-        # untimed warm-up (as the device leg has W warm-up steps): two
-        # host-built plans alive at once, as in the timed loop, so the
-        # library's memory pool has grown to hold both before timing starts
-        with tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[0], device=local,
-                        parents=args.parents, relabel=args.e2e_relabel) as hp0, \
-                tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[1], device=local,
-                           parents=args.parents, relabel=args.e2e_relabel) as hp1:
-            hp0.run_batch(mine[:1], lv_np, pa_np, stride=0)
-            hp1.run_batch(mine[:1], lv_np, pa_np, stride=0)
-        if dist:
-            dist.barrier()
-        torch.cuda.synchronize(dev)
-
         def make_plan(k):
             return tq.BfsPlan(rp_np, col_np, variant=args.variant, stream=streams[k % 2], device=local,
                               parents=args.parents, relabel=args.e2e_relabel)
 
+        def run_steps(n_steps, roots_):
+            """n_steps steps: step k runs every root on plan k (built from the
+            pinned host CSR) while a helper thread builds plan k+1."""
+            te, step_s = 0, []
+            nxt = make_plan(0)
+            for k in range(n_steps):
+                ts0 = time.perf_counter()
+                hp, box, th = nxt, {}, None
+                if k + 1 < n_steps:
+                    def build(k=k, box=box):
+                        try:
+                            box["plan"] = make_plan(k + 1)
+                        except Exception as ex:  # re-raised in the main thread
+                            box["error"] = ex
+                    th = threading.Thread(target=build)
+                    th.start()
+                # one C-ABI call per step: every root's level and parent arrays
+                # are copied to the (reused) pinned host buffers, D2H overlapped
+                # with the next root's BFS on a second stream
+                for s_ in hp.run_batch(roots_, lv_np, pa_np, stride=0):
+                    te += s_["traversed_edges"]
+                ts1 = time.perf_counter()
+                if th is not None:
+                    th.join()
+                    if "error" in box:
+                        raise box["error"]
+                    nxt = box["plan"]
+                ts2 = time.perf_counter()
+                hp.close()
+                step_s.append([round(ts1 - ts0, 3), round(ts2 - ts1, 3), round(time.perf_counter() - ts2, 3)])
+            return te, step_s
+
+        # untimed warm-up (as the device leg has W warm-up steps): three steps
+        # of the timed loop on 2 roots each, so that the library's memory pool
+        # has grown to the loop's peak (two plans alive, one being built)
+        run_steps(3, mine[:2])
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
-        te_e2e = 0
-        step_s = []
-        nxt = make_plan(0)
-        for k in range(args.steps):
-            ts0 = time.perf_counter()
-            hp, box, th = nxt, {}, None
-            if k + 1 < args.steps:
-                def build(k=k, box=box):
-                    try:
-                        box["plan"] = make_plan(k + 1)
-                    except Exception as ex:  # re-raised in the main thread
-                        box["error"] = ex
-                th = threading.Thread(target=build)
-                th.start()
-            # one C-ABI call per step: every root's level and parent arrays
-            # are copied to the (reused) pinned host buffers, D2H overlapped
-            # with the next root's BFS on a second stream
-            for s_ in hp.run_batch(mine, lv_np, pa_np, stride=0):
-                te_e2e += s_["traversed_edges"]
-            ts1 = time.perf_counter()
-            if th is not None:
-                th.join()
-                if "error" in box:
-                    raise box["error"]
-                nxt = box["plan"]
-            ts2 = time.perf_counter()
-            hp.close()
-            step_s.append([round(ts1 - ts0, 3), round(ts2 - ts1, 3), round(time.perf_counter() - ts2, 3)])
+        te_e2e, step_s = run_steps(args.steps, mine)
         torch.cuda.synchronize(dev)
         sec = time.perf_counter() - t0
         secv = torch.tensor([sec, te_e2e], dtype=torch.float64, device=coll_dev)
