@@ -613,10 +613,10 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     p->nnz = nnz;
 
     bool smem_auto_lanes = false;
-    // The plan's build work (graph upload, relabelling, chunk table) runs on
-    // an internal stream of the device's lowest priority, so that a plan
-    // built while another plan's BFS runs on a higher-priority stream yields
-    // the SMs to it (bench.py's e2e leg builds step k+1's plan during step k).
+    // The plan's build work (graph upload, chunk table) runs on an internal
+    // stream of the device's lowest priority, apart from the caller's stream
+    // (bench.py's e2e leg builds step k+1's plan during step k's BFS); the
+    // relabelling waits for the plan's first run (plan_relabel).
     cudaStream_t bs = nullptr;
     {
         int least = 0, greatest = 0;
