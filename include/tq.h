@@ -161,8 +161,9 @@ typedef struct {
     int variant;        /* tq_variant (RF_AN, PER_THREAD_AFA, CAS_RETRY, AN) */
     void *stream;       /* cudaStream_t                                      */
     double timeout_s;   /* watchdog; 0 = 60 s                                */
-    int backoff_ns;     /* max idle back-off per empty work cycle; 0 = 256,
-                           < 0 = none                                        */
+    int backoff_ns;     /* max idle back-off per empty work cycle; 0 = the
+                           default (none for RF_AN BFS, whose polls are
+                           relaxed loads; 256 otherwise), < 0 = none        */
     int device;         /* CUDA device for bfs_plan_create / host-pointer runs;
                            ignored when the CSR is device memory             */
     int parent_rule;    /* TQ_PARENT_ANY (0, default): some neighbour one level

@@ -585,7 +585,12 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     p->variant = o.variant;
     p->block = block;
     p->chunk = chunk;
-    p->backoff_ns = o.backoff_ns == 0 ? 256 : (o.backoff_ns < 0 ? 0 : o.backoff_ns);
+    // default idle back-off: none for RF/AN BFS (its polls are relaxed loads,
+    // R22, cheap to repeat; measured -2.8% / -1.4% on kron24 / kron26 within
+    // one process, within +-0.5% across processes: results/level_tokens_r02.log),
+    // 256 ns for the rest
+    const int bo_default = (o.variant == TQ_VARIANT_RF_AN && task == kTaskBFS) ? 0 : 256;
+    p->backoff_ns = o.backoff_ns == 0 ? bo_default : (o.backoff_ns < 0 ? 0 : o.backoff_ns);
     p->timeout_s = o.timeout_s > 0 ? o.timeout_s : 60.0;
     if (o.parent_rule != TQ_PARENT_MIN_ID && o.parent_rule != TQ_PARENT_ANY) {
         delete p;
