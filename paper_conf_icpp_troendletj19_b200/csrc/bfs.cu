@@ -35,13 +35,14 @@ constexpr int kWarps = kBlock / 32;
 // Staged tokens per warp (2-3 KiB smem). A larger stage publishes children in
 // bigger, later batches: fewer label-correcting re-scans, less work visible to
 // idle warps. Measured (results/ab_occupancy_r01.md, stage sweeps): 768 is best
-// for byte-mirror graphs (<= 2^25 vertices; kron24 3.87 -> 3.62 ms), 512 for
-// nibble-mirror ones (kron26 16.02 vs 16.27 ms).
+// for byte-mirror graphs (<= 2^25 vertices; kron24 3.87 -> 3.62 ms); 640 for
+// nibble-mirror ones (round 2, with 1,024-edge chunks: kron26 13.99 -> 13.73 ms
+// against 512, results/level_tokens_r02.log).
 // SSSP keeps 512, the setting it was tuned and validated with (its run-to-run
 // spread, 18.6-25.4 ms per s24 source at either size, hides any difference).
 template <int MIR, int TASK> __host__ __device__ constexpr int stage_cap()
 {
-    return (MIR == 8 && TASK == kTaskBFS) ? 768 : 512;
+    return TASK == kTaskBFS ? (MIR == 8 ? 768 : 640) : 512;
 }
 constexpr int kU = 4;                // 32-edge rounds in flight per lane
 // Resident blocks per SM requested from ptxas (40 warps/SM; <= 48 registers).
