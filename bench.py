@@ -447,6 +447,7 @@ def main():
     ap.add_argument("--no-configs", action="store_true", help="skip configs 1-4 (headline workload only)")
     ap.add_argument("--cpu-budget", type=float, default=20.0)
     ap.add_argument("--parents", default="any", choices=["any", "min_id"])
+    ap.add_argument("--chunk", type=int, default=0, help="bfs_opts.chunk of the device leg's plan (0 = default)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", 0))
@@ -498,7 +499,7 @@ def main():
 
     stream = torch.cuda.current_stream(dev)
     plan = tq.BfsPlan(row_ptr, col, variant=args.variant, stream=stream, device=local,
-                      parents=args.parents)
+                      parents=args.parents, chunk=args.chunk)
     level = torch.empty(n, dtype=torch.int32, device=dev)
     parent = torch.empty(n, dtype=torch.int32, device=dev)
 

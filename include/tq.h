@@ -156,9 +156,8 @@ typedef struct {
     int chunk;          /* sub-task size: max edges per task token (P:153
                            "a fixed number of uniformly complex sub-tasks";
                            P:159 fn3).  Vertices with more edges are split
-                           into chunk tokens.  0 = 512, or 1,024 on RF_AN
-                           BFS plans with the nibble mirror (see
-                           mirror_bits); power of 2 in [32, 2^16]           */
+                           into chunk tokens.  0 = 512; power of 2 in
+                           [32, 2^16]                                        */
     int variant;        /* tq_variant (RF_AN, PER_THREAD_AFA, CAS_RETRY, AN) */
     void *stream;       /* cudaStream_t                                      */
     double timeout_s;   /* watchdog; 0 = 60 s                                */

@@ -565,12 +565,10 @@ static tq_status plan_create_impl(const tq_csr *gph, const int32_t *weights, int
     if (o.variant < TQ_VARIANT_RF_AN || o.variant > TQ_VARIANT_AN) return TQ_ERR_UNSUPPORTED;
     if (task == kTaskSSSP && o.variant != TQ_VARIANT_RF_AN) return TQ_ERR_UNSUPPORTED;
     if (task == kTaskSSSP && nnz > 0 && !weights) return TQ_ERR_INVALID;
-    // default chunk: 512 edges; 1,024 where the plan will pick the nibble
-    // mirror (RF/AN BFS above 2^25 vertices, see below): kron26 -5%, while
-    // kron24 is 20% slower with 1,024 (results/level_tokens_r02.log)
-    const bool nibble_plan = task == kTaskBFS && o.variant == TQ_VARIANT_RF_AN &&
-                             (o.mirror_bits == 4 || (o.mirror_bits == 0 && n > (1ll << 25)));
-    int chunk = o.chunk ? o.chunk : (nibble_plan ? 1024 : 512);
+    // (default chunk 512: 1,024 looked 5% faster on 4 kron26 roots but is 6%
+    // slower over the bench's 64, and 20% slower on kron24;
+    // results/level_tokens_r02.log)
+    int chunk = o.chunk ? o.chunk : 512;
     if (chunk < 32 || chunk > 65536 || (chunk & (chunk - 1))) return TQ_ERR_INVALID;
     const int block = o.block ? o.block : 256;
     if (block != 256) return TQ_ERR_UNSUPPORTED;

@@ -36,8 +36,8 @@ constexpr int kWarps = kBlock / 32;
 // bigger, later batches: fewer label-correcting re-scans, less work visible to
 // idle warps. Measured (results/ab_occupancy_r01.md, stage sweeps): 768 is best
 // for byte-mirror graphs (<= 2^25 vertices; kron24 3.87 -> 3.62 ms); 640 for
-// nibble-mirror ones (round 2, with 1,024-edge chunks: kron26 13.99 -> 13.73 ms
-// against 512, results/level_tokens_r02.log).
+// nibble-mirror ones (round 2: kron26 over the bench's 64 roots 14.61 -> 14.43
+// ms together with no idle back-off, results/level_tokens_r02.log).
 // SSSP keeps 512, the setting it was tuned and validated with (its run-to-run
 // spread, 18.6-25.4 ms per s24 source at either size, hides any difference).
 template <int MIR, int TASK> __host__ __device__ constexpr int stage_cap()
