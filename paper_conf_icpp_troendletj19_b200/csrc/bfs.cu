@@ -117,7 +117,8 @@ __device__ __forceinline__ unsigned ld_cg_u8(const uint8_t *p, unsigned long lon
 // The byte mirror's probe through L1 (a weak load): stale-high values are all
 // the prefilter needs (R8), and with levels in the tokens (R22) no acquire
 // poll invalidates the L1, so the relabelled plan's top hubs (the first 2^14
-// ids, relabel.cu) stay cached there.  kron24: -3.5% (results/level_tokens_r02.log).
+// ids, relabel.cu) stay cached there.  kron24: -0.4% over the bench's batches, up to
+// -3.5% in per-root A/Bs (results/level_tokens_r02.log).
 __device__ __forceinline__ unsigned ld_l1_u8(const uint8_t *p, unsigned long long pol)
 {
     unsigned v;
